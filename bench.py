@@ -1,0 +1,379 @@
+#!/usr/bin/env python3
+"""Benchmark: GCUPS of the Smith-Waterman database search on B200 (BASELINE.json metric).
+
+One STEP = the whole hot path (profile build, both regimes, 32-bit recompute, scatter to
+caller order, and for N > 1 the NCCL score gather) for the 5 queries of config C2
+(lengths 144/375/729/1500/5478, BLOSUM62, gap open 10 / extend 2, threshold 3072) against
+a Swiss-Prot-shaped synthetic database of 540,000 sequences (~191M residues) PER GPU.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config C2|C1|C3]
+  python -m torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1 ... bench.py --gpus N
+
+value   = sum_q m_q * sum_j n_j (all ranks) / max-over-ranks device time of K steps (GCUPS);
+e2e     = same metric through the blocking host API (sw_search_batch: queries H2D, scores D2H);
+roofline= the fused search kernel (k_search) against the measured DPX-mix issue rate
+          (tools/int_peaks.cu -> MEASURED_INT_PEAKS.json), clock-normalised;
+cpu_baseline = the CPU oracle (oracle/, OpenMP, all host cores) on a bounded sample.
+--impl reference times that oracle as the reference arm (the paper ships no code).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from workloads import gen  # noqa: E402
+from workloads.matrices import MATRICES  # noqa: E402
+
+PAPER_CONTEXT = "PAPER.md: CUDASW++ 17 GCUPS (Tesla C1060, T=3072), >21 GCUPS with the improved kernel (C2050, TAIR)"
+
+
+def _env_int(k, d):
+    try:
+        return int(os.environ.get(k, d))
+    except ValueError:
+        return d
+
+
+# ------------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+        self.thread = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+            return
+        self.thread = threading.Thread(target=self._read, daemon=True)
+        self.thread.start()
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        if self.thread:
+            self.thread.join(timeout=2)
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            p = [x.strip() for x in ln.split(",")]
+            if len(p) < 7:
+                continue
+            try:
+                sm.append(float(p[0]))
+                mx = float(p[1])
+            except ValueError:
+                continue
+            for n, v in zip(names, p[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# ------------------------------------------------------------------------------- workload
+def make_workload(name: str, rank: int, world: int):
+    """Weak scaling: N ranks search N x (the config's database), one config-sized shard each."""
+    if name in ("C2", "C4"):
+        qs = [gen.make_query(L) for L in gen.C2_QUERY_LENGTHS]
+        lens = gen.sp_lengths(540_000 * world, seed=2)
+        seed, mat, T = 2, "BLOSUM62", 3072
+    elif name == "C1":
+        qs = [gen.make_query(144)]
+        lens = gen.sp_lengths(20_000 * world, seed=1)
+        seed, mat, T = 1, "BLOSUM62", 3072
+    elif name == "C3":
+        qs = [gen.make_query(L) for L in gen.C2_QUERY_LENGTHS]
+        lens = gen.long_lengths(4096 * world, seed=3)
+        seed, mat, T = 3, "BLOSUM62", 3072
+    else:
+        raise SystemExit(f"unknown config {name}")
+    sel = gen.shard_indices(lens, rank, world)
+    db = gen.build_database(lens, seed, qs, sel=sel)
+    return qs, db, lens, mat, 10, 2, T
+
+
+def cells_of(qs, total_residues):
+    return int(sum(int(q.size) for q in qs)) * int(total_residues)
+
+
+# ------------------------------------------------------------------------------- cpu oracle
+def oracle_sample(qs, db, budget_s: float, cores: int):
+    """Deterministic sample of the workload sized for ~budget_s of oracle time on `cores`."""
+    per_core = 0.30e9  # cells/s/core of the scalar oracle (SURVEY.md §8(d) measured 0.32-0.36)
+    target_cells = budget_s * per_core * cores
+    sum_m = sum(int(q.size) for q in qs)
+    target_res = max(1, int(target_cells / sum_m))
+    L = db.lengths
+    stride = max(1, int(db.total_residues // target_res))
+    idx = np.arange(0, db.num_seqs, stride)
+    sub_lens = L[idx]
+    off = np.concatenate([[0], np.cumsum(sub_lens)]).astype(np.int64)
+    res = np.concatenate([db.residues[db.offsets[i]:db.offsets[i + 1]] for i in idx]) if idx.size else \
+        np.zeros(0, np.uint8)
+    return idx, res, off, f"every {stride}-th sequence of the shard ({idx.size} seqs, {int(off[-1])} residues) x all queries"
+
+
+def run_oracle_step(qs, W, rho, sigma, res, off, threads):
+    import oracle
+    t0 = time.perf_counter()
+    for q in qs:
+        oracle.scores(q, W, rho, sigma, res, off, threads=threads)
+    return time.perf_counter() - t0
+
+
+def cpu_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
+# ------------------------------------------------------------------------------- reference arm
+def bench_reference(args, rank, world):
+    if rank != 0:
+        return
+    qs, db, _, mat, rho, sigma, T = make_workload(args.config, 0, 1)
+    W = MATRICES[mat]
+    cores = cpu_cores()
+    budget = max(1.0, 150.0 / max(1, args.steps + args.warmup))
+    idx, res, off, desc = oracle_sample(qs, db, budget, cores)
+    cells = cells_of(qs, int(off[-1]))
+    for _ in range(args.warmup):
+        run_oracle_step(qs, W, rho, sigma, res, off, cores)
+    times = [run_oracle_step(qs, W, rho, sigma, res, off, cores) for _ in range(args.steps)]
+    tot = sum(times)
+    gcups = cells * args.steps / tot / 1e9
+    line = {
+        "impl": "reference", "metric": "GCUPS", "value": round(gcups, 4), "unit": "GCUPS", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(1e3 * tot / args.steps, 3),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+        "config": {"workload": f"{args.config} oracle sample", "sample": desc, "queries": [int(q.size) for q in qs],
+                   "matrix": mat, "gap_open": rho, "gap_extend": sigma},
+        "cpu_baseline": {"value": round(gcups, 4), "unit": "GCUPS", "cores": cores, "kind": "oracle", "sample": desc},
+        "e2e": {"value": round(gcups, 4), "unit": "GCUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------------------- our arm
+def load_int_peaks():
+    p = os.path.join(ROOT, "MEASURED_INT_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f)
+    return None
+
+
+def bench_ours(args, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_hainscobr11_b200 as swp
+    from paper_conf_ipps_hainscobr11_b200 import build as swbuild
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    if rank == 0:
+        swbuild.build()
+    if world > 1:
+        dist.barrier()
+    qs, db, lens_all, mat, rho, sigma, T = make_workload(args.config, rank, world)
+    if args.threshold is not None:
+        T = args.threshold
+    W = MATRICES[mat]
+    nq = len(qs)
+    sw = swp.SmithWaterman(qs[0], W, rho, sigma)
+    sw.load_db(db.residues, db.offsets)
+    n_local = db.num_seqs
+    n_pad = int(-(-lens_all.shape[0] // world))  # ceil(N / world): uniform gather shard
+    scores = torch.zeros((nq, n_pad), dtype=torch.int32, device=dev)
+    gathered = torch.zeros((world, nq, n_pad), dtype=torch.int32, device=dev) if world > 1 else None
+    stream = torch.cuda.current_stream(dev)
+    sptr = stream.cuda_stream
+
+    cells_local = cells_of(qs, db.total_residues)
+    cells_total = cells_of(qs, int(lens_all.sum()))
+
+    def step():
+        # scores for query k land at scores[k, :n_local]
+        sw.search_batch_into(qs, scores.data_ptr(), T, sptr) if n_pad == n_local else \
+            _search_padded(sw, qs, scores, n_local, T, sptr)
+        if world > 1:
+            dist.all_gather_into_tensor(gathered, scores)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize(dev)
+    if world > 1:
+        dist.barrier()
+    clocks = ClockSampler(local_rank)
+    clocks.start()
+    time.sleep(0.3)
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    kern_ms = 0.0
+    rec_ms = 0.0
+    torch.cuda.synchronize(dev)
+    if world > 1:
+        dist.barrier()
+    ev0.record(stream)
+    for _ in range(args.steps):
+        step()
+    ev1.record(stream)
+    torch.cuda.synchronize(dev)
+    ms = ev0.elapsed_time(ev1)
+    # per-kernel device time of the dominant kernel (events on the launching streams), last step
+    km = sw.kernel_ms()
+    kern_ms, rec_ms = km["search_ms"], km["recompute_ms"]
+    st = sw.stats()
+    clk = clocks.stop()
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+
+    # end-to-end through the blocking host API (queries H2D, scores D2H), rank-local + max
+    e2e_steps = max(1, min(args.steps, 3))
+    t0 = time.perf_counter()
+    for _ in range(e2e_steps):
+        host = sw.search_batch(qs, T)
+        if world > 1:
+            dist.barrier()
+    e2e_s = (time.perf_counter() - t0) / e2e_steps
+    if world > 1:
+        t = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_s = float(t.item())
+    h2d = int(sum(int(q.size) for q in qs)) + 8 * (nq + 1)
+    d2h = int(host.size) * 4
+
+    if rank != 0:
+        sw.close()
+        if world > 1:
+            dist.destroy_process_group()
+        return
+    step_s = ms / 1e3 / args.steps
+    gcups = cells_total / step_s / 1e9
+    e2e_gcups = cells_total / e2e_s / 1e9
+
+    # roofline of the dominant kernel: the fused k_search launches of the last step
+    peaks = load_int_peaks()
+    achieved = cells_local / (kern_ms / 1e3) / 1e9 if kern_ms > 0 else None
+    roof = {"bound": "alu", "unit": "GCUPS", "achieved": round(achieved, 2) if achieved else None,
+            "peak": None, "frac": None, "traffic": None,
+            "kernel": "k_search (fused inter/intra-task), per-launch average over the 5 queries of the last step"}
+    if peaks and achieved:
+        f_mhz = clk.get("sm_mhz") or peaks.get("sm_mhz_during") or 1965.0
+        per_clk = peaks["cells_per_clk_per_gpu"]
+        peak = per_clk * f_mhz * 1e6 / 1e9
+        roof.update({"peak": round(peak, 1), "frac": round(achieved / peak, 4),
+                     "peak_basis": f"measured s16x2 cell-mix issue rate {per_clk:.1f} cells/clk/GPU "
+                                   f"(MEASURED_INT_PEAKS.json) x SM clock {f_mhz:.0f} MHz during the run"})
+    prof_path = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(prof_path):
+        try:
+            with open(prof_path) as f:
+                roof["traffic"] = json.load(f).get("k_search_dram_bytes_per_launch")
+        except Exception:
+            pass
+
+    # cpu baseline (oracle on a bounded sample), rank 0 at N == 1 only
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        cores = cpu_cores()
+        idx, res, off, desc = oracle_sample(qs, db, args.cpu_budget, cores)
+        ts = run_oracle_step(qs, W, rho, sigma, res, off, cores)
+        cpu = {"value": round(cells_of(qs, int(off[-1])) / ts / 1e9, 4), "unit": "GCUPS", "cores": cores,
+               "kind": "oracle", "sample": desc, "seconds": round(ts, 2)}
+
+    line = {
+        "metric": "GCUPS", "value": round(gcups, 2), "unit": "GCUPS", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(1e3 * step_s, 3), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "s16x2 (int32 recompute)", "data": "synthetic",
+        "config": {"workload": f"{args.config}: Swiss-Prot-shaped synthetic DB, 540k seqs / ~191M residues per GPU, "
+                               f"queries {[int(q.size) for q in qs]}", "matrix": mat, "gap_open": rho,
+                   "gap_extend": sigma, "threshold": T, "seqs_per_gpu": n_local,
+                   "residues_per_gpu": db.total_residues, "cells_per_step": cells_total,
+                   "l2": "inputs larger than L2 (device DB ~2x191 MB > 126 MB)", "parallelism": f"db-shard x{world}"},
+        "clocks": clk,
+        "e2e": {"value": round(e2e_gcups, 2), "unit": "GCUPS", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                "api": "sw_search_batch (blocking, host buffers; DB resident as in PAPER.md L32)"},
+        "gpu_launches": int(st["launches"]) * args.steps,
+        "roofline": roof,
+        "cpu_baseline": cpu,
+        "regimes": {"long_seqs": st["long_seqs"] // max(1, nq), "short_seqs": st["short_seqs"] // max(1, nq),
+                    "recomputed_s32": st["recomputed_s32"], "recompute_ms": round(rec_ms, 3)},
+        "paper_context": PAPER_CONTEXT,
+    }
+    print(json.dumps(line), flush=True)
+    sw.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def _search_padded(sw, qs, scores, n_local, T, sptr):
+    """Shard smaller than the uniform gather size: search into a contiguous [nq, n_local] view."""
+    import torch
+    tmp = getattr(_search_padded, "tmp", None)
+    if tmp is None or tmp.shape != (len(qs), n_local):
+        tmp = torch.zeros((len(qs), n_local), dtype=torch.int32, device=scores.device)
+        _search_padded.tmp = tmp
+    sw.search_batch_into(qs, tmp.data_ptr(), T, sptr)
+    scores[:, :n_local].copy_(tmp)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--threshold", type=int, default=None)
+    ap.add_argument("--cpu-budget", type=float, default=15.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    rank = _env_int("RANK", 0)
+    world = _env_int("WORLD_SIZE", 1)
+    local_rank = _env_int("LOCAL_RANK", 0)
+    if args.impl == "reference":
+        bench_reference(args, rank, world)
+        return
+    bench_ours(args, rank, world, local_rank)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,129 @@
+/*
+ * sw.h — C ABI of the B200-native Smith-Waterman database-search hot path
+ * (Hains, Cashero, Ottenberg, Bohm, Rajopadhye, "Improving CUDASW++", IPDPS 2011).
+ *
+ * The operation (PAPER.md L10 abstract; L12 §II Eq.(1); L14 §II-B): "computes the
+ * similarity scores of a query sequence paired with each sequence in a database".  For a
+ * query q (length m), database sequence d (length n), scoring function w, gap open rho and
+ * gap extension sigma, the score is max_{i,j} H[i][j] of
+ *
+ *     E[i][j] = max(E[i][j-1] - sigma, H[i][j-1] - rho)
+ *     F[i][j] = max(F[i-1][j] - sigma, H[i-1][j] - rho)
+ *     H[i][j] = max(0, E[i][j], F[i][j], H[i-1][j-1] + w(q_i, d_j))
+ *
+ * with H = 0 on row/column 0 and E/F = -inf there (readings c1-c4).  A gap of
+ * length k therefore costs rho + (k-1)*sigma (reading c2).  The result is exact (int32),
+ * identical for every length_threshold and every sharding (reading c8, c20).
+ *
+ * Conventions
+ *   - Every call returns an int status (SW_OK = 0); nothing aborts or exits.
+ *   - Residue / query codes are integers in [0, alphabet_size); the library never sees
+ *     letters.  matrix is row-major int8 [alphabet_size][alphabet_size], indexed
+ *     [query symbol][database symbol] (reading c5; it need not be symmetric).
+ *   - Ownership: the caller owns every input buffer; the library COPIES query, matrix and
+ *     database (device copies belong to the handle until sw_destroy).  Output buffers are
+ *     caller-allocated.
+ *   - A handle is bound to the CUDA device current at sw_create and is not thread-safe;
+ *     distinct handles may be used concurrently.  There is no CPU fallback: on a device
+ *     that is not compute capability 10.0 (sm_100a) sw_create returns SW_E_UNSUPPORTED.
+ */
+#ifndef SW_B200_H
+#define SW_B200_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct sw_handle_s* sw_handle;
+
+enum {
+  SW_OK = 0,
+  SW_E_INVALID = 1,      /* bad argument (NULL, length, code >= alphabet, bad offsets, ...) */
+  SW_E_STATE = 2,        /* call out of order (e.g. search before sw_load_db) */
+  SW_E_NOMEM = 3,        /* host or device allocation failed */
+  SW_E_CUDA = 4,         /* CUDA runtime error; detail in sw_last_error */
+  SW_E_UNSUPPORTED = 5   /* device is not sm_100 / parameters outside the supported range */
+};
+
+/* Limits (validated; SW_E_INVALID / SW_E_UNSUPPORTED otherwise). */
+#define SW_MAX_ALPHABET 32          /* alphabet_size in [1, 32] */
+#define SW_MAX_QUERY_LEN (1 << 16)  /* 1 <= query_len <= 65536 */
+#define SW_MAX_SEQ_LEN ((1 << 20) - 64)  /* every database sequence length <= 1,048,512 */
+
+/* Create a handle for one query and one scoring scheme (§II: q, w, rho, sigma).
+ *   query[query_len]      codes < alphabet_size, 1 <= query_len <= SW_MAX_QUERY_LEN
+ *   matrix[A*A]           int8, row = query symbol, column = database symbol
+ *   gap_open  (rho)       >= 0;  gap_extend (sigma) >= 0
+ * Supported range: gap_open + max(matrix) <= 127 and gap_open + gap_extend <= 32000
+ * (SW_E_UNSUPPORTED otherwise).
+ * Uploads the query and builds the query profile on the device (§II-A). */
+int sw_create(sw_handle* out, const uint8_t* query, int32_t query_len,
+              const int8_t* matrix, int32_t alphabet_size, int32_t gap_open, int32_t gap_extend);
+
+/* Replace the query (same matrix and penalties); keeps the loaded database. */
+int sw_set_query(sw_handle h, const uint8_t* query, int32_t query_len);
+
+/* Load a CSR database (copied): sequence k is residues[offsets[k] .. offsets[k+1]).
+ *   offsets[0] == 0, non-decreasing, offsets[num_seqs] == total_residues; each length
+ *   <= SW_MAX_SEQ_LEN; codes < alphabet_size; num_seqs >= 0 (length-0 sequences score 0).
+ * Host preprocessing (§II-C "sorted by length"): stable sort by length
+ * descending, pairing of neighbours, packing into the device layout.
+ * Replaces any previously loaded database. */
+int sw_load_db(sw_handle h, const uint8_t* residues, int64_t total_residues,
+               const int64_t* offsets, int64_t num_seqs);
+
+/* Score the handle's query against every database sequence (blocking).
+ *   scores_out: HOST int32[num_seqs], caller's database order.
+ *   length_threshold T >= 0: sequences with n >= T take the long-sequence (intra-task)
+ *   path, n < T the short-sequence (inter-task) path (§II-B: "If the
+ *   database sequence length is below 3072, the inter-task kernel is used. Otherwise,
+ *   the intra-task kernel is used.").  Scores do not depend on T. */
+int sw_search(sw_handle h, int32_t* scores_out, int32_t length_threshold);
+
+/* Same, stream-ordered: d_scores_out is a DEVICE int32[num_seqs] (e.g. a torch tensor);
+ * cuda_stream is a cudaStream_t (NULL = legacy default stream).  Returns after enqueueing. */
+int sw_search_async(sw_handle h, int32_t* d_scores_out, int32_t length_threshold, void* cuda_stream);
+
+/* Batch of queries against the loaded database (extension): query k is
+ * queries[q_offsets[k] .. q_offsets[k+1]); scores for query k go to
+ * d_scores_out[k*num_seqs .. (k+1)*num_seqs) (DEVICE pointer, stream-ordered).  The
+ * handle's own query is not changed.  Queries run concurrently on internal streams that
+ * are joined back into cuda_stream. */
+int sw_search_batch_async(sw_handle h, const uint8_t* queries, const int64_t* q_offsets,
+                          int32_t num_queries, int32_t* d_scores_out, int32_t length_threshold,
+                          void* cuda_stream);
+
+/* Host-pointer variant of sw_search_batch_async (blocking; host int32[num_queries*num_seqs]). */
+int sw_search_batch(sw_handle h, const uint8_t* queries, const int64_t* q_offsets,
+                    int32_t num_queries, int32_t* scores_out, int32_t length_threshold);
+
+/* Statistics of the last search on h (for measurement / tests):
+ *   out[0] = number of sequences recomputed in 32-bit after the 16-bit overflow flag,
+ *   out[1] = long-path (intra-task) sequences, out[2] = short-path sequences,
+ *   out[3] = kernel launches enqueued by the last search call. */
+int sw_last_stats(sw_handle h, int64_t out[4]);
+
+/* Device time of the last search call's kernels, from CUDA events recorded on the launching
+ * streams (valid after the work completed): out[0] = sum over queries of the search kernel
+ * (both regimes, one fused launch per query), out[1] = sum of the 32-bit recompute launches.
+ * Milliseconds. */
+int sw_last_kernel_ms(sw_handle h, double out[2]);
+
+/* Free everything (NULL-safe). */
+void sw_destroy(sw_handle h);
+
+/* Static text for a status code. */
+const char* sw_strerror(int status);
+
+/* Detail of the last failing call on h (never NULL; "" when none). */
+const char* sw_last_error(sw_handle h);
+
+/* Library / build identification, e.g. "sw_b200 sm_100a". */
+const char* sw_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SW_B200_H */

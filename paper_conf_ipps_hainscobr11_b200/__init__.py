@@ -1,0 +1,203 @@
+"""B200-native Smith-Waterman protein database search (Hains et al., "Improving CUDASW++",
+IPDPS 2011) — thin Python binding over the C ABI in include/sw.h.
+
+Argument marshalling only: every step of the search (profile build, both kernels, the
+32-bit recompute, the scatter to caller order) runs in libsw_b200.so on the GPU.  There is
+no CPU fallback: if the library is missing or the device is not sm_100a, calls raise.
+
+The function names mirror the C ABI: sw_create, sw_set_query, sw_load_db, sw_search,
+sw_search_async, sw_search_batch, sw_search_batch_async, sw_last_stats, sw_destroy.
+``SmithWaterman`` is a small object wrapper over the same calls.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libsw_b200.so")
+
+SW_OK, SW_E_INVALID, SW_E_STATE, SW_E_NOMEM, SW_E_CUDA, SW_E_UNSUPPORTED = range(6)
+EXPORTED = ["sw_create", "sw_set_query", "sw_load_db", "sw_search", "sw_search_async",
+            "sw_search_batch", "sw_search_batch_async", "sw_last_stats", "sw_last_kernel_ms", "sw_destroy",
+            "sw_strerror", "sw_last_error", "sw_version"]
+
+_lib = None
+
+
+class SWError(RuntimeError):
+    def __init__(self, status: int, detail: str = ""):
+        self.status = status
+        super().__init__(f"{_strerror(status)} (status {status}){': ' + detail if detail else ''}")
+
+
+def load_library(path: str = LIB_PATH):
+    """Load libsw_b200.so (raises if it has not been built: there is no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise ImportError(f"{path} not built; run `python -m paper_conf_ipps_hainscobr11_b200.build`")
+    L = ctypes.CDLL(path)
+    vp, i32, i64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64
+    L.sw_create.argtypes = [ctypes.POINTER(vp), vp, i32, vp, i32, i32, i32]
+    L.sw_set_query.argtypes = [vp, vp, i32]
+    L.sw_load_db.argtypes = [vp, vp, i64, vp, i64]
+    L.sw_search.argtypes = [vp, vp, i32]
+    L.sw_search_async.argtypes = [vp, vp, i32, vp]
+    L.sw_search_batch.argtypes = [vp, vp, vp, i32, vp, i32]
+    L.sw_search_batch_async.argtypes = [vp, vp, vp, i32, vp, i32, vp]
+    L.sw_last_stats.argtypes = [vp, vp]
+    L.sw_last_kernel_ms.argtypes = [vp, vp]
+    L.sw_destroy.argtypes = [vp]
+    L.sw_destroy.restype = None
+    L.sw_strerror.argtypes = [ctypes.c_int]
+    L.sw_strerror.restype = ctypes.c_char_p
+    L.sw_last_error.argtypes = [vp]
+    L.sw_last_error.restype = ctypes.c_char_p
+    L.sw_version.restype = ctypes.c_char_p
+    for name in ("sw_create", "sw_set_query", "sw_load_db", "sw_search", "sw_search_async", "sw_search_batch",
+                 "sw_search_batch_async", "sw_last_stats", "sw_last_kernel_ms"):
+        getattr(L, name).restype = ctypes.c_int
+    _lib = L
+    return L
+
+
+def _strerror(status: int) -> str:
+    try:
+        return load_library().sw_strerror(status).decode()
+    except ImportError:
+        return f"status {status}"
+
+
+def _check(h, status: int):
+    if status != SW_OK:
+        detail = load_library().sw_last_error(h).decode() if h else ""
+        raise SWError(status, detail)
+
+
+def _u8(a):
+    return np.ascontiguousarray(a, dtype=np.uint8)
+
+
+def sw_create(query, matrix, gap_open: int, gap_extend: int):
+    L = load_library()
+    q = _u8(query)
+    W = np.ascontiguousarray(matrix, dtype=np.int8)
+    h = ctypes.c_void_p()
+    _check(None, L.sw_create(ctypes.byref(h), q.ctypes.data, int(q.size), W.ctypes.data, int(W.shape[0]),
+                             int(gap_open), int(gap_extend)))
+    return h
+
+
+def sw_set_query(h, query):
+    q = _u8(query)
+    _check(h, load_library().sw_set_query(h, q.ctypes.data, int(q.size)))
+
+
+def sw_load_db(h, residues, offsets):
+    r = _u8(residues)
+    off = np.ascontiguousarray(offsets, dtype=np.int64)
+    rp = r.ctypes.data if r.size else None
+    _check(h, load_library().sw_load_db(h, rp, int(off[-1]), off.ctypes.data, int(off.size - 1)))
+
+
+def sw_search(h, num_seqs: int, length_threshold: int = 3072) -> np.ndarray:
+    out = np.zeros(max(num_seqs, 1), dtype=np.int32)
+    _check(h, load_library().sw_search(h, out.ctypes.data, int(length_threshold)))
+    return out[:num_seqs]
+
+
+def sw_search_async(h, d_scores_ptr: int, length_threshold: int, stream_ptr: int = 0):
+    _check(h, load_library().sw_search_async(h, ctypes.c_void_p(d_scores_ptr), int(length_threshold),
+                                             ctypes.c_void_p(stream_ptr)))
+
+
+def _batch(queries):
+    qs = [_u8(q) for q in queries]
+    off = np.zeros(len(qs) + 1, dtype=np.int64)
+    off[1:] = np.cumsum([q.size for q in qs])
+    cat = np.concatenate(qs) if qs else np.zeros(1, np.uint8)
+    return np.ascontiguousarray(cat), off
+
+
+def sw_search_batch(h, queries, num_seqs: int, length_threshold: int = 3072) -> np.ndarray:
+    cat, off = _batch(queries)
+    out = np.zeros((len(queries), max(num_seqs, 1)), dtype=np.int32)
+    _check(h, load_library().sw_search_batch(h, cat.ctypes.data, off.ctypes.data, len(queries), out.ctypes.data,
+                                              int(length_threshold)))
+    return out[:, :num_seqs]
+
+
+def sw_search_batch_async(h, queries, d_scores_ptr: int, length_threshold: int, stream_ptr: int = 0):
+    cat, off = _batch(queries)
+    _check(h, load_library().sw_search_batch_async(h, cat.ctypes.data, off.ctypes.data, len(queries),
+                                                   ctypes.c_void_p(d_scores_ptr), int(length_threshold),
+                                                   ctypes.c_void_p(stream_ptr)))
+
+
+def sw_last_stats(h) -> dict:
+    out = np.zeros(4, dtype=np.int64)
+    _check(h, load_library().sw_last_stats(h, out.ctypes.data))
+    return {"recomputed_s32": int(out[0]), "long_seqs": int(out[1]), "short_seqs": int(out[2]),
+            "launches": int(out[3])}
+
+
+def sw_last_kernel_ms(h) -> dict:
+    out = np.zeros(2, dtype=np.float64)
+    _check(h, load_library().sw_last_kernel_ms(h, out.ctypes.data))
+    return {"search_ms": float(out[0]), "recompute_ms": float(out[1])}
+
+
+def sw_destroy(h):
+    if h:
+        load_library().sw_destroy(h)
+
+
+class SmithWaterman:
+    """Object wrapper: one query + scoring scheme, one loaded database (caller order kept)."""
+
+    def __init__(self, query, matrix, gap_open: int, gap_extend: int):
+        self.h = sw_create(query, matrix, gap_open, gap_extend)
+        self.num_seqs = 0
+
+    def set_query(self, query):
+        sw_set_query(self.h, query)
+
+    def load_db(self, residues, offsets):
+        sw_load_db(self.h, residues, offsets)
+        self.num_seqs = int(np.asarray(offsets).shape[0] - 1)
+
+    def search(self, length_threshold: int = 3072) -> np.ndarray:
+        return sw_search(self.h, self.num_seqs, length_threshold)
+
+    def search_batch(self, queries, length_threshold: int = 3072) -> np.ndarray:
+        return sw_search_batch(self.h, queries, self.num_seqs, length_threshold)
+
+    def search_batch_into(self, queries, d_scores_ptr: int, length_threshold: int = 3072, stream_ptr: int = 0):
+        sw_search_batch_async(self.h, queries, d_scores_ptr, length_threshold, stream_ptr)
+
+    def stats(self) -> dict:
+        return sw_last_stats(self.h)
+
+    def kernel_ms(self) -> dict:
+        return sw_last_kernel_ms(self.h)
+
+    def close(self):
+        if self.h:
+            sw_destroy(self.h)
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

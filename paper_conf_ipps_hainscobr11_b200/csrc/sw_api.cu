@@ -1,0 +1,575 @@
+// sw_api.cu — the C ABI (include/sw.h): validation, host preprocessing of the database
+// (§II-C: "The database is sorted by length"), per-query planning and
+// stream-ordered launches of the sm_100a kernels.  No CPU fallback: every score is computed
+// by k_search (sw_engine.cuh) on the device.
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <numeric>
+#include <string>
+#include <vector>
+
+#include "../../include/sw.h"
+#include "sw_internal.h"
+
+using namespace swb;
+
+namespace {
+
+struct QuerySlot {
+  int cap_m = 0;
+  uint8_t* d_query = nullptr;
+  uint8_t* d_prof = nullptr;
+  size_t prof_cap = 0;
+  int32_t* d_work = nullptr;      // 4 counters
+  int32_t* d_ovf_count = nullptr;
+  int32_t* d_ovf_list = nullptr;
+  int64_t ovf_cap = 0;
+  uint2* d_rb_group = nullptr;
+  size_t rb_group_cap = 0;        // bytes
+  uint2* d_rb_team = nullptr;
+  size_t rb_team_cap = 0;
+  cudaStream_t stream = nullptr;
+  cudaEvent_t done = nullptr;
+};
+
+}  // namespace
+
+struct sw_handle_s {
+  int device = 0;
+  int num_sms = 0;
+  // scoring scheme
+  int A = 0, rho = 0, sigma = 0, max_w = 0, min_w = 0;
+  int8_t* d_matrix = nullptr;
+  std::vector<uint8_t> query;
+  // database
+  bool db_loaded = false;
+  int64_t n_seqs = 0;
+  int n_pairs = 0;
+  std::vector<int64_t> sorted_len;     // lengths in sorted (descending) order
+  std::vector<int32_t> h_pair_ncols;
+  uint16_t* d_cols = nullptr;
+  int64_t* d_pair_off = nullptr;
+  int32_t* d_pair_ncols = nullptr;
+  int32_t* d_perm = nullptr;
+  // scratch
+  std::vector<QuerySlot> slots;
+  int32_t* d_scores_tmp = nullptr;
+  int64_t scores_tmp_cap = 0;
+  uint8_t* d_batch_q = nullptr;
+  int64_t batch_q_cap = 0;
+  cudaEvent_t fork = nullptr;
+  // stats
+  int64_t stat_long = 0, stat_short = 0, stat_launches = 0;
+  int stat_nq = 0;
+  int32_t* h_ovf = nullptr;       // pinned, one overflow count per query of the last batch
+  int h_ovf_cap = 0;
+  std::vector<cudaEvent_t> ev;    // 3 per query: before search, after search, after recompute
+  std::string err;
+};
+
+namespace {
+
+int fail(sw_handle h, int code, const std::string& msg) {
+  if (h) h->err = msg;
+  return code;
+}
+
+int cuda_fail(sw_handle h, cudaError_t e, const char* what) {
+  std::string m = std::string(what) + ": " + cudaGetErrorName(e) + " (" + cudaGetErrorString(e) + ")";
+  if (h) h->err = m;
+  return e == cudaErrorMemoryAllocation ? SW_E_NOMEM : SW_E_CUDA;
+}
+
+#define SW_CUDA(h, call)                                   \
+  do {                                                     \
+    cudaError_t _e = (call);                               \
+    if (_e != cudaSuccess) return cuda_fail((h), _e, #call); \
+  } while (0)
+
+template <class T>
+int grow(sw_handle h, T** p, size_t* cap, size_t bytes, const char* what, cudaStream_t busy = nullptr) {
+  if (*cap >= bytes && *p) return SW_OK;
+  if (busy) cudaStreamSynchronize(busy);  // the old buffer may still be in use on this stream
+  if (*p) cudaFree(*p);
+  *p = nullptr;
+  *cap = 0;
+  if (bytes == 0) return SW_OK;
+  cudaError_t e = cudaMalloc(reinterpret_cast<void**>(p), bytes);
+  if (e != cudaSuccess) return cuda_fail(h, e, what);
+  *cap = bytes;
+  return SW_OK;
+}
+
+int64_t round_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
+
+// ------------------------------------------------------------------------------------ planning
+struct Plan {
+  KernelConfig cfg;
+  int short_passes, long_passes, team_warps;
+  int m_pad, pstride, prof_bytes;
+  // s32 recompute
+  KernelConfig rcfg;
+  int r_passes, r_team_warps;
+  int grid, rgrid;
+};
+
+int team_warps_for(int passes) {
+  if (passes <= 1) return 1;
+  const int rounds = (passes + kWarps - 1) / kWarps;
+  return (passes + rounds - 1) / rounds;
+}
+
+// Pick the menu entry minimising the estimated issue cost: padded rows x (1 + per-step
+// overhead / per-step cell work) for each regime, weighted by the regime's residue share.
+int make_plan(sw_handle h, int m, double long_frac, Plan* pl) {
+  const int A1 = h->A + 1;
+  double best = 1e300;
+  int best_i = -1;
+  for (int i = 0; i < menu_size(); ++i) {
+    const KernelConfig c = menu_entry(i);
+    if (c.lane != 0) continue;
+    const int rs = c.G * c.Rs, rl = 32 * c.Rl;
+    const int ps = (m + rs - 1) / rs, plong = (m + rl - 1) / rl;
+    const int rpass = (m + 32 * 16 - 1) / (32 * 16);
+    const int m_pad = std::max({ps * rs, plong * rl, rpass * 32 * 16});
+    const int64_t bytes = (int64_t)A1 * round_up(m_pad, 16);
+    if (bytes > 200 * 1024) continue;
+    const double cs = (double)ps * rs * (1.0 + 22.0 / (6.5 * c.Rs)) * (1.0 + (c.G - 1) / (ps * 350.0));
+    const double cl = (double)plong * rl * (1.0 + 22.0 / (6.5 * c.Rl));
+    const double cost = cs * (1.0 - long_frac) + cl * long_frac;
+    if (cost < best) { best = cost; best_i = i; }
+  }
+  // test hooks: force a menu entry / team size (used by the parity tests to cover every
+  // compiled configuration; never needed for correctness)
+  if (const char* f = getenv("SW_FORCE_MENU")) {
+    const int i = atoi(f);
+    if (i >= 0 && i < menu_size() && menu_entry(i).lane == 0) best_i = i;
+  }
+  if (best_i < 0) return fail(h, SW_E_UNSUPPORTED, "query profile does not fit in shared memory (query_len * (alphabet_size + 1) too large)");
+  const KernelConfig c = menu_entry(best_i);
+  pl->cfg = c;
+  pl->short_passes = (m + c.G * c.Rs - 1) / (c.G * c.Rs);
+  pl->long_passes = (m + 32 * c.Rl - 1) / (32 * c.Rl);
+  pl->team_warps = team_warps_for(pl->long_passes);
+  if (const char* f = getenv("SW_FORCE_TEAM_WARPS")) {
+    const int w = atoi(f);
+    if (w >= 1 && w <= kWarps) pl->team_warps = std::min(w, std::max(1, pl->long_passes));
+  }
+  pl->rcfg = recompute_config();
+  pl->r_passes = (m + 32 * pl->rcfg.Rl - 1) / (32 * pl->rcfg.Rl);
+  pl->r_team_warps = team_warps_for(pl->r_passes);
+  pl->m_pad = std::max({pl->short_passes * c.G * c.Rs, pl->long_passes * 32 * c.Rl, pl->r_passes * 32 * pl->rcfg.Rl});
+  pl->pstride = (int)round_up(pl->m_pad, 16);
+  pl->prof_bytes = A1 * pl->pstride;
+  int bps = 0;
+  cudaError_t e = configure_kernel(c, pl->prof_bytes, &bps);
+  if (e != cudaSuccess) return cuda_fail(h, e, "configure search kernel");
+  if (bps < 1) return fail(h, SW_E_UNSUPPORTED, "search kernel cannot be resident");
+  pl->grid = bps * h->num_sms;
+  e = configure_kernel(pl->rcfg, pl->prof_bytes, &bps);
+  if (e != cudaSuccess) return cuda_fail(h, e, "configure recompute kernel");
+  if (bps < 1) return fail(h, SW_E_UNSUPPORTED, "recompute kernel cannot be resident");
+  pl->rgrid = bps * h->num_sms;
+  return SW_OK;
+}
+
+int ensure_slots(sw_handle h, int n) {
+  while ((int)h->slots.size() < n) {
+    QuerySlot s;
+    SW_CUDA(h, cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking));
+    SW_CUDA(h, cudaEventCreateWithFlags(&s.done, cudaEventDisableTiming));
+    SW_CUDA(h, cudaMalloc(&s.d_work, 4 * sizeof(int32_t)));
+    SW_CUDA(h, cudaMalloc(&s.d_ovf_count, sizeof(int32_t)));
+    h->slots.push_back(s);
+  }
+  return SW_OK;
+}
+
+int validate_query(sw_handle h, const uint8_t* q, int32_t m) {
+  if (!q) return fail(h, SW_E_INVALID, "query is NULL");
+  if (m <= 0 || m > SW_MAX_QUERY_LEN) return fail(h, SW_E_INVALID, "query_len out of range [1, 65536]");
+  for (int32_t i = 0; i < m; ++i)
+    if (q[i] >= h->A) return fail(h, SW_E_INVALID, "query code >= alphabet_size at position " + std::to_string(i));
+  return SW_OK;
+}
+
+// Enqueue one query (device query pointer) on slot s; scores to d_out (device, caller order).
+int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t* d_out, int32_t T,
+                  int32_t* h_ovf, cudaEvent_t* ev) {
+  // regime split: sorted_len is descending; long = n >= T (§II-B)
+  const int64_t n_long_seqs =
+      std::lower_bound(h->sorted_len.begin(), h->sorted_len.end(), (int64_t)T, std::greater_equal<int64_t>()) -
+      h->sorted_len.begin();
+  const int n_long = (int)((n_long_seqs + 1) / 2);
+  int64_t long_cols = 0, all_cols = 0;
+  for (int p = 0; p < h->n_pairs; ++p) {
+    all_cols += h->h_pair_ncols[p];
+    if (p < n_long) long_cols += h->h_pair_ncols[p];
+  }
+  const double long_frac = all_cols ? (double)long_cols / (double)all_cols : 0.0;
+  Plan pl;
+  int rc = make_plan(h, m, long_frac, &pl);
+  if (rc) return rc;
+
+  // scratch: profile, overflow list, row buffers
+  rc = grow(h, &s.d_prof, &s.prof_cap, (size_t)pl.prof_bytes, "alloc profile", s.stream);
+  if (rc) return rc;
+  size_t ovf_bytes = (size_t)std::max<int64_t>(h->n_seqs, 1) * sizeof(int32_t);
+  size_t ovf_cap = (size_t)s.ovf_cap * sizeof(int32_t);
+  rc = grow(h, &s.d_ovf_list, &ovf_cap, ovf_bytes, "alloc overflow list", s.stream);
+  if (rc) return rc;
+  s.ovf_cap = (int64_t)(ovf_cap / sizeof(int32_t));
+  const int64_t max_cols_all = h->n_pairs ? h->h_pair_ncols[0] : 0;
+  const int64_t max_cols_short = (n_long < h->n_pairs) ? h->h_pair_ncols[n_long] : 0;
+  const int G = pl.cfg.G;
+  size_t rbg = 0;
+  if (pl.short_passes > 1 && max_cols_short > 0)
+    rbg = (size_t)pl.grid * kWarps * (32 / G) * max_cols_short * sizeof(uint2);
+  size_t rbt = 0;
+  if (pl.long_passes > 1 && n_long > 0) {
+    const int nteams = kWarps / pl.team_warps;
+    rbt = (size_t)pl.grid * nteams * (pl.team_warps + 1) * h->h_pair_ncols[0] * sizeof(uint2);
+  }
+  if (pl.r_passes > 1) {
+    const int nteams = kWarps / pl.r_team_warps;
+    rbt = std::max(rbt, (size_t)pl.rgrid * nteams * (pl.r_team_warps + 1) * max_cols_all * sizeof(uint2));
+  }
+  rc = grow(h, &s.d_rb_group, &s.rb_group_cap, rbg, "alloc group row buffers", s.stream);
+  if (rc) return rc;
+  rc = grow(h, &s.d_rb_team, &s.rb_team_cap, rbt, "alloc team row buffers", s.stream);
+  if (rc) return rc;
+
+  cudaStream_t st = s.stream;
+  SW_CUDA(h, cudaMemsetAsync(s.d_work, 0, 4 * sizeof(int32_t), st));
+  SW_CUDA(h, cudaMemsetAsync(s.d_ovf_count, 0, sizeof(int32_t), st));
+  SW_CUDA(h, launch_profile(s.d_prof, d_q, m, h->d_matrix, h->A, h->rho, pl.pstride, st));
+
+  SearchParams p{};
+  p.prof = s.d_prof;
+  p.pstride = pl.pstride;
+  p.prof_bytes = pl.prof_bytes;
+  p.pad_letter = h->A;
+  p.rho = h->rho;
+  p.sigma = h->sigma;
+  p.max_w = h->max_w;
+  p.cols = h->d_cols;
+  p.pair_off = h->d_pair_off;
+  p.pair_ncols = h->d_pair_ncols;
+  p.n_pairs = h->n_pairs;
+  p.n_seqs = (int)h->n_seqs;
+  p.perm = h->d_perm;
+  p.scores = d_out;
+  p.n_long = n_long;
+  p.item_list = nullptr;
+  p.item_count = nullptr;
+  p.work = s.d_work;
+  p.ovf_list = s.d_ovf_list;
+  p.ovf_count = s.d_ovf_count;
+  p.short_passes = pl.short_passes;
+  p.long_passes = pl.long_passes;
+  p.team_warps = pl.team_warps;
+  p.rb_group = s.d_rb_group;
+  p.rb_group_cols = max_cols_short;
+  p.rb_team = s.d_rb_team;
+  p.rb_team_cols = max_cols_all;
+  SW_CUDA(h, cudaEventRecord(ev[0], st));
+  SW_CUDA(h, launch_search(pl.cfg, p, pl.grid, pl.prof_bytes, st));
+  SW_CUDA(h, cudaEventRecord(ev[1], st));
+
+  // exact 32-bit recompute of sequences whose 16-bit best reached 32767 - max_w
+  SearchParams r = p;
+  r.item_list = s.d_ovf_list;
+  r.item_count = s.d_ovf_count;
+  r.work = s.d_work + 2;
+  r.long_passes = pl.r_passes;
+  r.team_warps = pl.r_team_warps;
+  SW_CUDA(h, launch_search(pl.rcfg, r, pl.rgrid, pl.prof_bytes, st));
+  SW_CUDA(h, cudaEventRecord(ev[2], st));
+  SW_CUDA(h, cudaMemcpyAsync(h_ovf, s.d_ovf_count, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+
+  h->stat_long += n_long_seqs;
+  h->stat_short += h->n_seqs - n_long_seqs;
+  h->stat_launches += 3;
+  return SW_OK;
+}
+
+int run_batch(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq, int32_t* d_out, int32_t T,
+              cudaStream_t user) {
+  h->stat_long = h->stat_short = h->stat_launches = 0;
+  h->stat_nq = nq;
+  if (h->n_seqs == 0 || nq == 0) return SW_OK;
+  int rc = ensure_slots(h, std::min(nq, 4));
+  if (rc) return rc;
+  if (h->h_ovf_cap < nq) {
+    if (h->h_ovf) { cudaDeviceSynchronize(); cudaFreeHost(h->h_ovf); }
+    h->h_ovf = nullptr;
+    h->h_ovf_cap = 0;
+    SW_CUDA(h, cudaMallocHost(&h->h_ovf, (size_t)nq * sizeof(int32_t)));
+    h->h_ovf_cap = nq;
+  }
+  memset(h->h_ovf, 0, (size_t)nq * sizeof(int32_t));
+  while ((int)h->ev.size() < 3 * nq) {
+    cudaEvent_t e;
+    SW_CUDA(h, cudaEventCreate(&e));
+    h->ev.push_back(e);
+  }
+  const int ns = std::min(nq, 4);
+  SW_CUDA(h, cudaEventRecord(h->fork, user));
+  for (int k = 0; k < ns; ++k) SW_CUDA(h, cudaStreamWaitEvent(h->slots[k].stream, h->fork, 0));
+  for (int k = 0; k < nq; ++k) {
+    QuerySlot& s = h->slots[k % ns];
+    rc = enqueue_query(h, s, d_queries + qoff[k], (int)(qoff[k + 1] - qoff[k]), d_out + (int64_t)k * h->n_seqs, T,
+                       h->h_ovf + k, h->ev.data() + 3 * k);
+    if (rc) return rc;
+  }
+  for (int k = 0; k < ns; ++k) {
+    SW_CUDA(h, cudaEventRecord(h->slots[k].done, h->slots[k].stream));
+    SW_CUDA(h, cudaStreamWaitEvent(user, h->slots[k].done, 0));
+  }
+  return SW_OK;
+}
+
+}  // namespace
+
+// ============================================================================ C ABI
+extern "C" {
+
+const char* sw_strerror(int status) {
+  switch (status) {
+    case SW_OK: return "ok";
+    case SW_E_INVALID: return "invalid argument";
+    case SW_E_STATE: return "call out of order";
+    case SW_E_NOMEM: return "out of memory";
+    case SW_E_CUDA: return "CUDA error";
+    case SW_E_UNSUPPORTED: return "unsupported device or parameters";
+    default: return "unknown status";
+  }
+}
+
+const char* sw_last_error(sw_handle h) { return h ? h->err.c_str() : ""; }
+
+const char* sw_version(void) { return "sw_b200 1.0 sm_100a"; }
+
+int sw_create(sw_handle* out, const uint8_t* query, int32_t query_len, const int8_t* matrix, int32_t alphabet_size,
+              int32_t gap_open, int32_t gap_extend) {
+  if (!out) return SW_E_INVALID;
+  *out = nullptr;
+  if (!matrix || alphabet_size < 1 || alphabet_size > SW_MAX_ALPHABET) return SW_E_INVALID;
+  if (gap_open < 0 || gap_extend < 0) return SW_E_INVALID;
+  sw_handle h = new (std::nothrow) sw_handle_s();
+  if (!h) return SW_E_NOMEM;
+  h->A = alphabet_size;
+  h->rho = gap_open;
+  h->sigma = gap_extend;
+  h->max_w = -128;
+  h->min_w = 127;
+  for (int i = 0; i < alphabet_size * alphabet_size; ++i) {
+    h->max_w = std::max<int>(h->max_w, matrix[i]);
+    h->min_w = std::min<int>(h->min_w, matrix[i]);
+  }
+  int rc = validate_query(h, query, query_len);
+  if (rc) { delete h; return rc; }
+  if (gap_open + std::max(h->max_w, 0) > 127 || (int64_t)gap_open + gap_extend > 32000) {
+    delete h;
+    return SW_E_UNSUPPORTED;
+  }
+  cudaError_t e = cudaGetDevice(&h->device);
+  cudaDeviceProp prop;
+  if (e == cudaSuccess) e = cudaGetDeviceProperties(&prop, h->device);
+  if (e != cudaSuccess) { delete h; return SW_E_UNSUPPORTED; }
+  if (!(prop.major == 10 && prop.minor == 0)) { delete h; return SW_E_UNSUPPORTED; }
+  h->num_sms = prop.multiProcessorCount;
+  if (cudaMalloc(&h->d_matrix, (size_t)alphabet_size * alphabet_size) != cudaSuccess ||
+      cudaMemcpy(h->d_matrix, matrix, (size_t)alphabet_size * alphabet_size, cudaMemcpyHostToDevice) != cudaSuccess ||
+      cudaEventCreateWithFlags(&h->fork, cudaEventDisableTiming) != cudaSuccess) {
+    sw_destroy(h);
+    return SW_E_CUDA;
+  }
+  h->query.assign(query, query + query_len);
+  *out = h;
+  return SW_OK;
+}
+
+int sw_set_query(sw_handle h, const uint8_t* query, int32_t query_len) {
+  if (!h) return SW_E_INVALID;
+  int rc = validate_query(h, query, query_len);
+  if (rc) return rc;
+  h->query.assign(query, query + query_len);
+  return SW_OK;
+}
+
+int sw_load_db(sw_handle h, const uint8_t* residues, int64_t total_residues, const int64_t* offsets,
+               int64_t num_seqs) {
+  if (!h) return SW_E_INVALID;
+  if (num_seqs < 0 || total_residues < 0) return fail(h, SW_E_INVALID, "negative size");
+  if (num_seqs > (int64_t)0x7ffffffe) return fail(h, SW_E_INVALID, "num_seqs too large");
+  if (!offsets) return fail(h, SW_E_INVALID, "offsets is NULL");
+  if (total_residues > 0 && !residues) return fail(h, SW_E_INVALID, "residues is NULL");
+  if (offsets[0] != 0 || offsets[num_seqs] != total_residues)
+    return fail(h, SW_E_INVALID, "offsets[0] must be 0 and offsets[num_seqs] == total_residues");
+  std::vector<int64_t> len((size_t)num_seqs);
+  for (int64_t k = 0; k < num_seqs; ++k) {
+    len[k] = offsets[k + 1] - offsets[k];
+    if (len[k] < 0) return fail(h, SW_E_INVALID, "offsets not non-decreasing at " + std::to_string(k));
+    if (len[k] > SW_MAX_SEQ_LEN) return fail(h, SW_E_INVALID, "sequence longer than SW_MAX_SEQ_LEN at " + std::to_string(k));
+  }
+  for (int64_t t = 0; t < total_residues; ++t)
+    if (residues[t] >= h->A) return fail(h, SW_E_INVALID, "residue code >= alphabet_size at " + std::to_string(t));
+
+  // free the previous database
+  cudaFree(h->d_cols); cudaFree(h->d_pair_off); cudaFree(h->d_pair_ncols); cudaFree(h->d_perm);
+  h->d_cols = nullptr; h->d_pair_off = nullptr; h->d_pair_ncols = nullptr; h->d_perm = nullptr;
+  h->db_loaded = false;
+
+  // stable sort by length, descending (ties keep input order)
+  std::vector<int32_t> perm((size_t)num_seqs);
+  std::iota(perm.begin(), perm.end(), 0);
+  std::stable_sort(perm.begin(), perm.end(), [&](int32_t a, int32_t b) { return len[a] > len[b]; });
+  h->sorted_len.resize((size_t)num_seqs);
+  for (int64_t k = 0; k < num_seqs; ++k) h->sorted_len[k] = len[perm[k]];
+  const int n_pairs = (int)((num_seqs + 1) / 2);
+  std::vector<int64_t> pair_off((size_t)n_pairs + 1, 0);
+  h->h_pair_ncols.assign((size_t)n_pairs, 0);
+  for (int p = 0; p < n_pairs; ++p) {
+    const int64_t lo = h->sorted_len[2 * p];
+    const int64_t hi = (2 * p + 1 < num_seqs) ? h->sorted_len[2 * p + 1] : 0;
+    const int64_t nc = round_up(std::max<int64_t>({lo, hi, (int64_t)kMinCols}), kColAlign);
+    h->h_pair_ncols[p] = (int32_t)nc;
+    pair_off[p + 1] = pair_off[p] + nc;
+  }
+  const int64_t total_cols = pair_off[n_pairs];
+  std::vector<uint16_t> cols((size_t)std::max<int64_t>(total_cols, 1));
+  const uint16_t pad = (uint16_t)h->A;
+  for (int p = 0; p < n_pairs; ++p) {
+    uint16_t* dst = cols.data() + pair_off[p];
+    const int64_t nc = h->h_pair_ncols[p];
+    const int64_t s0 = perm[2 * p];
+    const int64_t l0 = len[s0];
+    const uint8_t* r0 = residues ? residues + offsets[s0] : nullptr;
+    const bool has1 = 2 * p + 1 < num_seqs;
+    const int64_t s1 = has1 ? perm[2 * p + 1] : 0;
+    const int64_t l1 = has1 ? len[s1] : 0;
+    const uint8_t* r1 = (has1 && residues) ? residues + offsets[s1] : nullptr;
+    for (int64_t j = 0; j < nc; ++j) {
+      const uint16_t a = j < l0 ? r0[j] : pad;
+      const uint16_t b = j < l1 ? r1[j] : pad;
+      dst[j] = (uint16_t)(a | (b << 8));
+    }
+  }
+  h->n_seqs = num_seqs;
+  h->n_pairs = n_pairs;
+  if (num_seqs == 0) { h->db_loaded = true; return SW_OK; }
+  SW_CUDA(h, cudaMalloc(&h->d_cols, cols.size() * sizeof(uint16_t)));
+  SW_CUDA(h, cudaMalloc(&h->d_pair_off, (size_t)n_pairs * sizeof(int64_t)));
+  SW_CUDA(h, cudaMalloc(&h->d_pair_ncols, (size_t)n_pairs * sizeof(int32_t)));
+  SW_CUDA(h, cudaMalloc(&h->d_perm, (size_t)num_seqs * sizeof(int32_t)));
+  SW_CUDA(h, cudaMemcpy(h->d_cols, cols.data(), cols.size() * sizeof(uint16_t), cudaMemcpyHostToDevice));
+  SW_CUDA(h, cudaMemcpy(h->d_pair_off, pair_off.data(), (size_t)n_pairs * sizeof(int64_t), cudaMemcpyHostToDevice));
+  SW_CUDA(h, cudaMemcpy(h->d_pair_ncols, h->h_pair_ncols.data(), (size_t)n_pairs * sizeof(int32_t), cudaMemcpyHostToDevice));
+  SW_CUDA(h, cudaMemcpy(h->d_perm, perm.data(), (size_t)num_seqs * sizeof(int32_t), cudaMemcpyHostToDevice));
+  h->db_loaded = true;
+  return SW_OK;
+}
+
+int sw_search_batch_async(sw_handle h, const uint8_t* queries, const int64_t* q_offsets, int32_t num_queries,
+                          int32_t* d_scores_out, int32_t length_threshold, void* cuda_stream) {
+  if (!h) return SW_E_INVALID;
+  if (!h->db_loaded) return fail(h, SW_E_STATE, "sw_load_db has not been called");
+  if (num_queries < 0 || !q_offsets || (num_queries > 0 && !queries)) return fail(h, SW_E_INVALID, "bad query batch");
+  if (length_threshold < 0) return fail(h, SW_E_INVALID, "length_threshold < 0");
+  if (h->n_seqs > 0 && num_queries > 0 && !d_scores_out) return fail(h, SW_E_INVALID, "d_scores_out is NULL");
+  if (q_offsets[0] != 0) return fail(h, SW_E_INVALID, "q_offsets[0] != 0");
+  for (int k = 0; k < num_queries; ++k) {
+    const int64_t m = q_offsets[k + 1] - q_offsets[k];
+    if (m <= 0 || m > SW_MAX_QUERY_LEN) return fail(h, SW_E_INVALID, "query length out of range in batch");
+    int rc = validate_query(h, queries + q_offsets[k], (int32_t)m);
+    if (rc) return rc;
+  }
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(cuda_stream);
+  const int64_t tot = q_offsets[num_queries];
+  size_t cap = (size_t)h->batch_q_cap;
+  int rc = grow(h, &h->d_batch_q, &cap, (size_t)std::max<int64_t>(tot, 1), "alloc batch queries");
+  if (rc) return rc;
+  h->batch_q_cap = (int64_t)cap;
+  if (tot > 0) SW_CUDA(h, cudaMemcpyAsync(h->d_batch_q, queries, (size_t)tot, cudaMemcpyHostToDevice, st));
+  return run_batch(h, h->d_batch_q, q_offsets, num_queries, d_scores_out, length_threshold, st);
+}
+
+int sw_search_async(sw_handle h, int32_t* d_scores_out, int32_t length_threshold, void* cuda_stream) {
+  if (!h) return SW_E_INVALID;
+  const int64_t qo[2] = {0, (int64_t)h->query.size()};
+  return sw_search_batch_async(h, h->query.data(), qo, 1, d_scores_out, length_threshold, cuda_stream);
+}
+
+int sw_search_batch(sw_handle h, const uint8_t* queries, const int64_t* q_offsets, int32_t num_queries,
+                    int32_t* scores_out, int32_t length_threshold) {
+  if (!h) return SW_E_INVALID;
+  if (!h->db_loaded) return fail(h, SW_E_STATE, "sw_load_db has not been called");
+  if (num_queries < 0) return fail(h, SW_E_INVALID, "num_queries < 0");
+  const int64_t need = (int64_t)num_queries * h->n_seqs;
+  if (need > 0 && !scores_out) return fail(h, SW_E_INVALID, "scores_out is NULL");
+  size_t cap = (size_t)h->scores_tmp_cap * sizeof(int32_t);
+  int rc = grow(h, &h->d_scores_tmp, &cap, (size_t)std::max<int64_t>(need, 1) * sizeof(int32_t), "alloc scores");
+  if (rc) return rc;
+  h->scores_tmp_cap = (int64_t)(cap / sizeof(int32_t));
+  rc = sw_search_batch_async(h, queries, q_offsets, num_queries, h->d_scores_tmp, length_threshold, nullptr);
+  if (rc) return rc;
+  if (need > 0)
+    SW_CUDA(h, cudaMemcpy(scores_out, h->d_scores_tmp, (size_t)need * sizeof(int32_t), cudaMemcpyDeviceToHost));
+  SW_CUDA(h, cudaDeviceSynchronize());
+  return SW_OK;
+}
+
+int sw_search(sw_handle h, int32_t* scores_out, int32_t length_threshold) {
+  if (!h) return SW_E_INVALID;
+  const int64_t qo[2] = {0, (int64_t)h->query.size()};
+  return sw_search_batch(h, h->query.data(), qo, 1, scores_out, length_threshold);
+}
+
+int sw_last_stats(sw_handle h, int64_t out[4]) {
+  if (!h || !out) return SW_E_INVALID;
+  int64_t ovf = 0;
+  // valid once the last search's stream work has completed
+  for (int k = 0; k < std::min(h->stat_nq, h->h_ovf_cap); ++k) ovf += h->h_ovf[k];
+  out[0] = ovf;
+  out[1] = h->stat_long;
+  out[2] = h->stat_short;
+  out[3] = h->stat_launches;
+  return SW_OK;
+}
+
+int sw_last_kernel_ms(sw_handle h, double out[2]) {
+  if (!h || !out) return SW_E_INVALID;
+  out[0] = out[1] = 0.0;
+  for (int k = 0; k < h->stat_nq && 3 * k + 2 < (int)h->ev.size(); ++k) {
+    float a = 0.f, b = 0.f;
+    cudaError_t e = cudaEventElapsedTime(&a, h->ev[3 * k], h->ev[3 * k + 1]);
+    if (e == cudaSuccess) e = cudaEventElapsedTime(&b, h->ev[3 * k + 1], h->ev[3 * k + 2]);
+    if (e != cudaSuccess) return cuda_fail(h, e, "cudaEventElapsedTime");
+    out[0] += a;
+    out[1] += b;
+  }
+  return SW_OK;
+}
+
+void sw_destroy(sw_handle h) {
+  if (!h) return;
+  for (cudaEvent_t e : h->ev) cudaEventDestroy(e);
+  for (QuerySlot& s : h->slots) {
+    if (s.stream) cudaStreamSynchronize(s.stream);
+    cudaFree(s.d_prof); cudaFree(s.d_work); cudaFree(s.d_ovf_count); cudaFree(s.d_ovf_list);
+    cudaFree(s.d_rb_group); cudaFree(s.d_rb_team); cudaFree(s.d_query);
+    if (s.stream) cudaStreamDestroy(s.stream);
+    if (s.done) cudaEventDestroy(s.done);
+  }
+  cudaFree(h->d_matrix); cudaFree(h->d_cols); cudaFree(h->d_pair_off); cudaFree(h->d_pair_ncols);
+  cudaFree(h->d_perm); cudaFree(h->d_scores_tmp); cudaFree(h->d_batch_q);
+  if (h->fork) cudaEventDestroy(h->fork);
+  if (h->h_ovf) cudaFreeHost(h->h_ovf);
+  delete h;
+}
+
+}  // extern "C"

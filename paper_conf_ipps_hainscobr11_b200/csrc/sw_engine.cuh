@@ -1,0 +1,428 @@
+// sw_engine.cuh — the sm_100a Smith-Waterman engine.
+//
+// What every lane computes is Eq.(1) of PAPER.md (L12 §II):
+//   E[i][j] = max(E[i][j-1] - sigma, H[i][j-1] - rho)
+//   F[i][j] = max(F[i-1][j] - sigma, H[i-1][j] - rho)
+//   H[i][j] = max(0, E[i][j], F[i][j], H[i-1][j-1] + w(q_i, d_j))
+// in the "hr" form used here: registers hold hr = H - rho, so that the single value hr
+// feeds both E of the right neighbour and F of the lower neighbour, and the query profile
+// stores w + rho so that H = max(hr_diag + (w + rho), E, F, 0) is one fused DPX op.
+//
+// Work decomposition (B200 design, not the paper's; §III is prior art):
+//   * a CHAIN is GC consecutive lanes of a warp; lane l owns R consecutive query rows of
+//     the current strip (strip = GC*R rows, "a set of n_th * t_height rows
+//     as a strip") and sweeps the database columns; lane l processes column j one step
+//     after lane l-1, receiving (H-rho, F) of the row above through __shfl_up_sync
+//     (registers for horizontal, shuffles for vertical/diagonal dependencies — the
+//     paper's registers + shared memory split);
+//   * strips are chained with a full row buffer of (H-rho, F) per column in global/L2
+//     ("the bottom row of a strip must be saved for the next pass", L18-L20) and the lane
+//     that finishes a strip moves straight on to the next one: one pipeline fill/flush per
+//     alignment (future work item iii of PAPER.md L30 §VI);
+//   * GROUP mode (inter-task, short sequences): GC = G <= 32 lanes per database pair,
+//     several pairs per warp, persistent warps pull pairs longest-first;
+//   * TEAM mode (intra-task, long sequences, §II-B.2 and L18 §III): a team of
+//     W warps per database pair; warp w of the team takes strips w, w+W, ...; strip
+//     hand-off through the row buffers with shared-memory progress flags (acquire/release);
+//   * two database sequences share one 32-bit register as signed 16-bit lanes (LaneS16x2,
+//     DPX VIADDMNMX/VIMNMX3) with an exact overflow flag; flagged sequences are recomputed
+//     with 32-bit lanes (LaneS32) by the same engine.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "sw_internal.h"
+
+namespace swb {
+
+#define SWB_FULL 0xffffffffu
+
+// PRMT with a compile-time selector.  Inline PTX because __byte_perm keeps only 3 bits per
+// selector nibble, while the 4th bit (sign replication of the selected byte) is what turns
+// the int8 profile entries into sign-extended 16/32-bit lanes in one instruction.
+template <uint32_t SEL>
+__device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b) {
+  uint32_t d;
+  asm("prmt.b32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "n"(SEL));
+  return d;
+}
+
+// ------------------------------------------------------------------------------------ lanes
+struct LaneS16x2 {
+  static constexpr int kSeqs = 2;
+  static __device__ __forceinline__ uint32_t splat(int v) { return ((uint32_t)v & 0xffffu) * 0x10001u; }
+  // max(a - sigma, b): E / F update (a = E or F, nsig = -sigma, b = hr of left / upper cell)
+  static __device__ __forceinline__ uint32_t gap(uint32_t a, uint32_t nsig, uint32_t b) {
+    return __viaddmax_s16x2(a, nsig, b);
+  }
+  static __device__ __forceinline__ uint32_t max2(uint32_t a, uint32_t b) { return __vmaxs2(a, b); }
+  // H = max(hr_diag + (w + rho), max(E, F), 0)
+  static __device__ __forceinline__ uint32_t hcell(uint32_t d, uint32_t w, uint32_t ef) {
+    return __viaddmax_s16x2_relu(d, w, ef);
+  }
+  static __device__ __forceinline__ uint32_t add(uint32_t a, uint32_t b) { return __vadd2(a, b); }
+  static __device__ __forceinline__ uint32_t max3(uint32_t a, uint32_t b, uint32_t c) {
+    return __vimax3_s16x2(a, b, c);
+  }
+  // substitution value of profile row k (of a 4-row int8 word) for both sequences,
+  // sign-extended to two s16 halves with one PRMT
+  template <int K>
+  static __device__ __forceinline__ uint32_t subst(uint32_t wlo, uint32_t whi) {
+    return prmt<0xC480u + K * 0x1111u>(wlo, whi);
+  }
+};
+
+struct LaneS32 {
+  static constexpr int kSeqs = 1;
+  static __device__ __forceinline__ uint32_t splat(int v) { return (uint32_t)v; }
+  static __device__ __forceinline__ uint32_t gap(uint32_t a, uint32_t nsig, uint32_t b) {
+    return (uint32_t)__viaddmax_s32((int)a, (int)nsig, (int)b);
+  }
+  static __device__ __forceinline__ uint32_t max2(uint32_t a, uint32_t b) { return (uint32_t)max((int)a, (int)b); }
+  static __device__ __forceinline__ uint32_t hcell(uint32_t d, uint32_t w, uint32_t ef) {
+    return (uint32_t)__viaddmax_s32_relu((int)d, (int)w, (int)ef);
+  }
+  static __device__ __forceinline__ uint32_t add(uint32_t a, uint32_t b) { return a + b; }
+  static __device__ __forceinline__ uint32_t max3(uint32_t a, uint32_t b, uint32_t c) {
+    return (uint32_t)__vimax3_s32((int)a, (int)b, (int)c);
+  }
+  template <int K>
+  static __device__ __forceinline__ uint32_t subst(uint32_t wlo, uint32_t) {
+    return prmt<0x8880u + K * 0x1111u>(wlo, 0u);
+  }
+};
+
+// ------------------------------------------------------------------------------------ PTX helpers
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+// TMA bulk copy global -> shared (cp.async.bulk, completes on the mbarrier)
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
+  asm volatile(
+      "{\n"
+      ".reg .pred P1;\n"
+      "WAIT_LOOP:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+      "@!P1 bra WAIT_LOOP;\n"
+      "}\n" ::"r"(smem_u32(bar)),
+      "r"(phase)
+      : "memory");
+}
+__device__ __forceinline__ uint32_t ld_acquire_smem(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.cta.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_smem(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.cta.shared::cta.u32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
+}
+__device__ __forceinline__ void team_bar(int team, int W) {
+  if (W > 1) {
+    asm volatile("bar.sync %0, %1;" ::"r"(team + 1), "r"(W * 32) : "memory");
+  } else {
+    __syncwarp();
+  }
+}
+
+// R bytes of one profile letter row -> R/4 words (4 query rows per word, §III-B
+// "stores the similarity scores of four symbols in a single variable")
+template <int R>
+__device__ __forceinline__ void load_prof(uint32_t (&w)[R / 4], const uint8_t* p) {
+  if constexpr (R % 16 == 0) {
+#pragma unroll
+    for (int i = 0; i < R / 16; ++i) {
+      const uint4 v = reinterpret_cast<const uint4*>(p)[i];
+      w[4 * i + 0] = v.x; w[4 * i + 1] = v.y; w[4 * i + 2] = v.z; w[4 * i + 3] = v.w;
+    }
+  } else if constexpr (R % 8 == 0) {
+#pragma unroll
+    for (int i = 0; i < R / 8; ++i) {
+      const uint2 v = reinterpret_cast<const uint2*>(p)[i];
+      w[2 * i + 0] = v.x; w[2 * i + 1] = v.y;
+    }
+  } else {
+#pragma unroll
+    for (int i = 0; i < R / 4; ++i) w[i] = reinterpret_cast<const uint32_t*>(p)[i];
+  }
+}
+
+__device__ __forceinline__ uint32_t pass_tag(int pass, int cols_done) {
+  return ((uint32_t)pass << 20) | (uint32_t)cols_done;
+}
+
+struct ChainConst {
+  const uint8_t* sprof;   // shared-memory profile
+  int pstride;
+  int rho, sigma;
+  uint32_t padpair;       // residue pair of two pad letters
+};
+
+// One chain of GC lanes sweeping `steps` pipeline steps over its passes (see file header).
+// Returns this lane's running best (packed per Lane).
+template <class L, int GC, int R, bool TEAM>
+__device__ __forceinline__ uint32_t run_chain(const ChainConst& c, const uint16_t* __restrict__ cols, int ncols,
+                                              int half, int steps, int pass0, int pstep, int npass,
+                                              int passes_total, uint2* __restrict__ rb, int64_t rb_cols,
+                                              int rb_nslot, uint32_t* prog) {
+  static_assert(R % 4 == 0 && R % 2 == 0, "R must be a multiple of 4");
+  const int lane = threadIdx.x & 31;
+  const int gl = lane & (GC - 1);
+  const uint32_t nrho = L::splat(-c.rho);
+  const uint32_t nsig = L::splat(-c.sigma);
+  const int hshift = 8 * half;
+
+  uint32_t hr[R], e[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) { hr[r] = nrho; e[r] = nrho; }
+  uint32_t best = 0, hrdiag0 = nrho;
+  uint32_t y_hr = nrho, y_f = nrho, y_res = c.padpair;
+  int col = -gl, k = 0, P = pass0;
+  const uint8_t* prow = c.sprof;  // row window of this lane in the profile (set at column 0)
+
+  // lane 0 of the chain streams residues and the previous strip's bottom row, one step ahead
+  uint32_t in_res = c.padpair, in_hr = nrho, in_f = nrho;
+  auto fetch = [&](int fk, int fcol, int fP) {
+    in_res = c.padpair; in_hr = nrho; in_f = nrho;
+    if (fk < npass) {
+      in_res = cols[fcol];
+      if (fP > 0) {
+        const int slot = TEAM ? ((fP - 1) % rb_nslot) : 0;
+        if (TEAM && (fcol & 7) == 0) {
+          const uint32_t need = pass_tag(fP - 1, fcol + 8);
+          while (ld_acquire_smem(prog + slot) < need) __nanosleep(20);
+        }
+        const uint2 v = rb[slot * rb_cols + fcol];
+        in_hr = v.x; in_f = v.y;
+      }
+    }
+  };
+  if (gl == 0) fetch(0, 0, pass0);
+
+  for (int s = 0; s < steps; ++s) {
+    uint32_t x_hr = __shfl_up_sync(SWB_FULL, y_hr, 1, GC);
+    uint32_t x_f = __shfl_up_sync(SWB_FULL, y_f, 1, GC);
+    uint32_t x_res = __shfl_up_sync(SWB_FULL, y_res, 1, GC);
+    if (gl == 0) { x_hr = in_hr; x_f = in_f; x_res = in_res; }
+    if (col == 0) {
+      // first column of a strip: H[i][0] = 0 (hr = -rho), E[i][0] = -inf (reading c4: any
+      // value <= 0 gives the same H; -rho is used), diagonal of row 0 is H[r0-1][0] = 0.
+#pragma unroll
+      for (int r = 0; r < R; ++r) { hr[r] = nrho; e[r] = nrho; }
+      hrdiag0 = nrho;
+      // past the last strip the lane only sees pad columns: keep the window in bounds
+      prow = c.sprof + (k < npass ? (P * GC + gl) * R : 0);
+    }
+    // query-profile words for the two letters of this column
+    uint32_t wlo[R / 4], whi[R / 4];
+    {
+      const int alo = (x_res >> hshift) & 0xff;
+      load_prof<R>(wlo, prow + alo * c.pstride);
+      if constexpr (L::kSeqs == 2) {
+        const int ahi = x_res >> 8;
+        load_prof<R>(whi, prow + ahi * c.pstride);
+      }
+    }
+    uint32_t hrup = x_hr, f = x_f, hrdiag = hrdiag0, hprev = 0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      uint32_t wv;
+      const uint32_t a = wlo[r >> 2];
+      const uint32_t b = (L::kSeqs == 2) ? whi[r >> 2] : 0u;
+      switch (r & 3) {
+        case 0: wv = L::template subst<0>(a, b); break;
+        case 1: wv = L::template subst<1>(a, b); break;
+        case 2: wv = L::template subst<2>(a, b); break;
+        default: wv = L::template subst<3>(a, b); break;
+      }
+      e[r] = L::gap(e[r], nsig, hr[r]);          // E[i][j] = max(E[i][j-1] - sigma, H[i][j-1] - rho)
+      f = L::gap(f, nsig, hrup);                 // F[i][j] = max(F[i-1][j] - sigma, H[i-1][j] - rho)
+      const uint32_t ef = L::max2(e[r], f);
+      const uint32_t h = L::hcell(hrdiag, wv, ef);  // max(H[i-1][j-1] + w, E, F, 0)
+      hrdiag = hr[r];
+      hr[r] = L::add(h, nrho);                   // H - rho
+      hrup = hr[r];
+      if (r & 1) best = L::max3(best, hprev, h); else hprev = h;
+    }
+    hrdiag0 = x_hr;
+    y_hr = hrup; y_f = f; y_res = x_res;
+
+    // last lane: save the strip's bottom row for the next strip (not after the last strip)
+    if (gl == GC - 1 && col >= 0 && k < npass && P < passes_total - 1) {
+      const int slot = TEAM ? (P % rb_nslot) : 0;
+      rb[slot * rb_cols + col] = make_uint2(y_hr, y_f);
+      if (TEAM && ((col & 7) == 7 || col == ncols - 1)) {
+        __threadfence_block();
+        st_release_smem(prog + slot, pass_tag(P, col + 1));
+      }
+    }
+    // lane 0: prefetch the next step's inputs
+    if (gl == 0) {
+      int nk = k, ncol = col + 1, nP = P;
+      if (ncol == ncols) { ncol = 0; ++nk; nP += pstep; }
+      fetch(nk, ncol, nP);
+    }
+    ++col;
+    if (col == ncols) { col = 0; ++k; P += pstep; }
+    if (!TEAM) __syncwarp();
+  }
+  return best;
+}
+
+// emit the score(s) of one chain result; s16x2: both sequences of the pair
+template <class L>
+__device__ __forceinline__ void emit(const SearchParams& p, uint32_t b, int pair, int half) {
+  if constexpr (L::kSeqs == 2) {
+    const int limit = 32767 - p.max_w;
+    const int s0 = 2 * pair, s1 = 2 * pair + 1;
+    const int lo = (int)(int16_t)(b & 0xffffu), hi = (int)(int16_t)(b >> 16);
+    if (lo >= limit) p.ovf_list[atomicAdd(p.ovf_count, 1)] = s0; else p.scores[p.perm[s0]] = lo;
+    if (s1 < p.n_seqs) {
+      if (hi >= limit) p.ovf_list[atomicAdd(p.ovf_count, 1)] = s1; else p.scores[p.perm[s1]] = hi;
+    }
+  } else {
+    const int s = 2 * pair + half;
+    p.scores[p.perm[s]] = (int)b;
+  }
+}
+
+template <class L, int G, int Rs, int Rl>
+__global__ void __launch_bounds__(kThreads, 1) k_search(const SearchParams p) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  __shared__ __align__(8) uint64_t mbar;
+  __shared__ uint32_t sprog[2 * kWarps];
+  __shared__ uint32_t sred[kWarps];
+  __shared__ int32_t sitem[kWarps];
+
+  // ---- stage the query profile in shared memory with TMA bulk copies (§III-B:
+  //      the profile lives in texture memory there; on sm_100a it is smem-resident)
+  if (threadIdx.x == 0) {
+    mbar_init(&mbar, 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    mbar_expect_tx(&mbar, (uint32_t)p.prof_bytes);
+    constexpr int kChunk = 32768;
+    for (int off = 0; off < p.prof_bytes; off += kChunk) {
+      const int sz = min(kChunk, p.prof_bytes - off);
+      bulk_g2s(smem + off, p.prof + off, (uint32_t)sz, &mbar);
+    }
+  }
+  mbar_wait(&mbar, 0);
+
+  ChainConst c;
+  c.sprof = smem;
+  c.pstride = p.pstride;
+  c.rho = p.rho;
+  c.sigma = p.sigma;
+  c.padpair = (uint32_t)p.pad_letter | ((uint32_t)p.pad_letter << 8);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+  // ---- phase 1: TEAM (intra-task) items — long sequences, or the 32-bit recompute list
+  {
+    const int W = p.team_warps;
+    const int nteams = kWarps / W;
+    const int team = warp / W, wt = warp % W;
+    if (team < nteams) {
+      uint32_t* prog = sprog + team * (W + 1);
+      const int n_items = p.item_list ? *p.item_count : p.n_long;
+      for (;;) {
+        team_bar(team, W);
+        if (wt == 0 && lane == 0) {
+          sitem[team] = atomicAdd(&p.work[0], 1);
+          for (int i = 0; i <= W; ++i) prog[i] = 0u;
+        }
+        team_bar(team, W);
+        const int item = sitem[team];
+        if (item >= n_items) break;
+        int pair = item, half = 0;
+        if (p.item_list) {
+          const int sq = p.item_list[item];
+          pair = sq >> 1;
+          half = sq & 1;
+        }
+        const int ncols = p.pair_ncols[pair];
+        const uint16_t* cp = p.cols + p.pair_off[pair];
+        uint2* rb = p.rb_team + ((int64_t)(blockIdx.x * nteams + team) * (W + 1)) * p.rb_team_cols;
+        // One strip per chain sweep (fill + flush per strip).  A warp must not start strip
+        // P + W before all its lanes finished strip P: its lane 0 may wait for strip P + W - 1,
+        // which transitively needs the tail of strip P (deadlock for short rows otherwise).
+        uint32_t b = 0;
+        for (int P = wt; P < p.long_passes; P += W) {
+          const uint32_t bp = run_chain<L, 32, Rl, true>(c, cp, ncols, half, ncols + 31, P, W, 1, p.long_passes,
+                                                         rb, p.rb_team_cols, W + 1, prog);
+          b = L::max2(b, bp);
+        }
+#pragma unroll
+        for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
+        if (lane == 0) sred[warp] = b;
+        team_bar(team, W);
+        if (wt == 0 && lane == 0) {
+          uint32_t bb = sred[team * W];
+          for (int i = 1; i < W; ++i) bb = L::max2(bb, sred[team * W + i]);
+          emit<L>(p, bb, pair, half);
+        }
+      }
+    }
+  }
+
+  // ---- phase 2: GROUP (inter-task) items — short sequences, G lanes per pair
+  if (p.item_list == nullptr) {
+    constexpr int GPW = 32 / G;
+    const int gi = lane / G, gl = lane & (G - 1);
+    const int nshort = p.n_pairs - p.n_long;
+    for (;;) {
+      int base = 0;
+      if (lane == 0) base = atomicAdd(&p.work[1], GPW);
+      base = __shfl_sync(SWB_FULL, base, 0);
+      if (base >= nshort) break;
+      const bool valid = base + gi < nshort;
+      const int pair = p.n_long + base + gi;
+      const int ncols = valid ? p.pair_ncols[pair] : 0;
+      const uint16_t* cp = p.cols + (valid ? p.pair_off[pair] : 0);
+      const int npass = valid ? p.short_passes : 0;
+      const int steps = (int)__reduce_max_sync(SWB_FULL, (unsigned)(npass * ncols)) + G - 1;
+      uint2* rb = p.rb_group + ((int64_t)(blockIdx.x * kWarps + warp) * GPW + gi) * p.rb_group_cols;
+      uint32_t b = run_chain<L, G, Rs, false>(c, cp, ncols, 0, steps, 0, 1, npass, p.short_passes, rb,
+                                              p.rb_group_cols, 1, nullptr);
+#pragma unroll
+      for (int o = G / 2; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
+      if (gl == 0 && valid) emit<L>(p, b, pair, 0);
+    }
+  }
+}
+
+template <class L, int G, int Rs, int Rl>
+cudaError_t launch_search_t(const SearchParams& p, int grid, int smem_bytes, cudaStream_t st) {
+  k_search<L, G, Rs, Rl><<<grid, kThreads, smem_bytes, st>>>(p);
+  return cudaGetLastError();
+}
+
+template <class L, int G, int Rs, int Rl>
+cudaError_t configure_t(int smem_bytes, int* blocks_per_sm) {
+  cudaError_t e = cudaFuncSetAttribute(k_search<L, G, Rs, Rl>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       smem_bytes);
+  if (e != cudaSuccess) return e;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search<L, G, Rs, Rl>, kThreads,
+                                                       smem_bytes);
+}
+
+}  // namespace swb

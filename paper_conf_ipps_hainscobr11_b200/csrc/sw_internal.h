@@ -1,0 +1,72 @@
+// sw_internal.h — shared between the host side (sw_api.cu) and the kernel instantiations.
+// Not part of the public ABI (include/sw.h is).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace swb {
+
+constexpr int kThreads = 512;            // threads per CTA (16 warps)
+constexpr int kWarps = kThreads / 32;
+constexpr int kMinCols = 48;             // every pair is padded to >= 48 columns (>= G + 16)
+constexpr int kColAlign = 8;             // pair column counts are multiples of 8 (16 bytes)
+constexpr int kPadValue = -128;          // profile value of pad letters / pad query rows
+
+// One persistent search launch for one query.
+struct SearchParams {
+  // query profile P[a][i] = w(q_i, a) + rho as int8 (a < A), row A = pad; i < m_pad
+  const uint8_t* prof;       // global, (A + 1) * pstride bytes
+  int pstride;               // bytes per letter row (multiple of 16, >= m_pad)
+  int prof_bytes;            // (A + 1) * pstride
+  int pad_letter;            // == A
+  int rho, sigma, max_w;
+  // database, sorted by length descending and paired (2p, 2p+1)
+  const uint16_t* cols;      // interleaved columns: cols[pair_off[p] + j] = d_lo[j] | d_hi[j] << 8
+  const int64_t* pair_off;   // in u16 units
+  const int32_t* pair_ncols; // padded column count n' (multiple of 8, >= kMinCols)
+  int n_pairs;
+  int n_seqs;
+  const int32_t* perm;       // sorted position -> caller index
+  int32_t* scores;           // caller order, int32
+  // work partition: items [0, n_long) run in team (intra-task) mode, [n_long, n_pairs) in
+  // group (inter-task) mode.  For the 32-bit recompute kernel items come from item_list.
+  int n_long;
+  const int32_t* item_list;  // s32 recompute: sorted sequence positions (nullptr otherwise)
+  const int32_t* item_count; // s32 recompute: device count
+  int32_t* work;             // [0] team-item counter, [1] group-item counter
+  int32_t* ovf_list;         // sequences whose 16-bit best may have wrapped
+  int32_t* ovf_count;
+  // passes over the query: group mode G*R_s rows per pass, team mode 32*R_l rows per pass
+  int short_passes;
+  int long_passes;
+  int team_warps;            // warps per team (1..kWarps), teams = kWarps / team_warps
+  // row buffers (strip bottom rows, §III "the bottom row of a strip must
+  // be saved for the next pass"), uint2 = (H - rho, F) per column
+  uint2* rb_group; int64_t rb_group_cols;   // per group slot
+  uint2* rb_team;  int64_t rb_team_cols;    // per (team slot, pass mod (team_warps+1))
+};
+
+// Kernel configuration menu entry: G lanes x R_s rows in group mode, 32 lanes x R_l rows
+// in team mode.  Lane = 0 (s16x2, two sequences per register) or 1 (s32, one sequence).
+struct KernelConfig {
+  int lane;
+  int G;
+  int Rs;
+  int Rl;
+};
+
+// Launch one search; returns the CUDA error of the launch.
+cudaError_t launch_search(const KernelConfig& cfg, const SearchParams& p, int grid, int smem_bytes,
+                          cudaStream_t st);
+// Max dynamic smem / occupancy helpers for a config.
+cudaError_t configure_kernel(const KernelConfig& cfg, int smem_bytes, int* blocks_per_sm);
+// The menu of compiled configurations.
+int menu_size();
+KernelConfig menu_entry(int i);
+KernelConfig recompute_config();
+
+// Profile build: prof[a][i] = (i < m && a < A) ? W[q_i][a] + rho : -128.
+cudaError_t launch_profile(uint8_t* prof, const uint8_t* q, int m, const int8_t* W, int A, int rho,
+                           int pstride, cudaStream_t st);
+
+}  // namespace swb

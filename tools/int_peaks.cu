@@ -45,33 +45,60 @@ __global__ void __launch_bounds__(512) k_peak(uint32_t* out, uint32_t seed, long
   if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
 }
 
-// The s16x2 Smith-Waterman cell mix exactly as the kernels issue it
-// (per row: PRMT + VIADDMNMX x2 + VIMNMX + VIADDMNMX.RELU + VIADD + 0.5 VIMNMX3).
+// The s16x2 Smith-Waterman cell update exactly as sw_engine.cuh issues it (per row: PRMT +
+// VIADDMNMX x2 + VIMNMX + VIADDMNMX.RELU + VIADD + 0.5 VIMNMX3), profile words varying per
+// column, no memory traffic: the ALU speed of light of the engine's arithmetic.
+template <uint32_t SEL>
+__device__ __forceinline__ uint32_t prmt_imm(uint32_t a, uint32_t b) {
+  uint32_t d;
+  asm("prmt.b32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "n"(SEL));
+  return d;
+}
+constexpr int CM_R = 16;
 __global__ void __launch_bounds__(512) k_cellmix(uint32_t* out, uint32_t seed, long long* cyc) {
-  constexpr int R = 16;
+  constexpr int R = CM_R;
   uint32_t hr[R], e[R];
 #pragma unroll
-  for (int r = 0; r < R; ++r) { hr[r] = seed + r; e[r] = seed * 3 + r; }
-  uint32_t best = 0, hrup0 = seed, f0 = seed * 7;
+  for (int r = 0; r < R; ++r) { hr[r] = 0xFFF6FFF6u; e[r] = 0xFFF6FFF6u; }
+  uint32_t best = 0, hrup0 = 0xFFF6FFF6u, f0 = 0xFFF6FFF6u, hrdiag0 = 0xFFF6FFF6u;
   const uint32_t nsig = 0xFFFEFFFEu, nrho = 0xFFF6FFF6u;
-  uint32_t p0 = seed * 0x01010101u, p1 = seed * 0x02020202u;
+  // profile rows in shared memory, read with LDS.128 exactly like the engine (25 letters)
+  __shared__ __align__(16) uint32_t sprof[25 * R];
+  for (int i = threadIdx.x; i < 25 * R; i += blockDim.x) sprof[i] = (seed + i) * 0x01010101u;
+  __syncthreads();
+  uint32_t res = threadIdx.x * 7u + seed;
   long long t0 = clock64();
   for (int it = 0; it < ITERS / 8; ++it) {
-    uint32_t hrup = hrup0 ^ it, f = f0, hrdiag = hrup0;
-    uint32_t hprev = 0;
+    uint32_t wlo[R / 4], whi[R / 4];
+    const uint4* plo = reinterpret_cast<const uint4*>(sprof + (res & 15) * R);
+    const uint4* phi = reinterpret_cast<const uint4*>(sprof + ((res >> 4) & 15) * R);
+#pragma unroll
+    for (int k = 0; k < R / 16; ++k) {
+      const uint4 a = plo[k], b = phi[k];
+      wlo[4 * k] = a.x; wlo[4 * k + 1] = a.y; wlo[4 * k + 2] = a.z; wlo[4 * k + 3] = a.w;
+      whi[4 * k] = b.x; whi[4 * k + 1] = b.y; whi[4 * k + 2] = b.z; whi[4 * k + 3] = b.w;
+    }
+    res = res * 0x9E37u + 0x79B9u;
+    uint32_t hrup = hrup0, f = f0, hrdiag = hrdiag0, hprev = 0;
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-      uint32_t w = __byte_perm(p0 + it, p1, 0xC480 + (r & 3) * 0x1111);
+      uint32_t w;
+      switch (r & 3) {
+        case 0: w = prmt_imm<0xC480u>(wlo[r >> 2], whi[r >> 2]); break;
+        case 1: w = prmt_imm<0xD591u>(wlo[r >> 2], whi[r >> 2]); break;
+        case 2: w = prmt_imm<0xE6A2u>(wlo[r >> 2], whi[r >> 2]); break;
+        default: w = prmt_imm<0xF7B3u>(wlo[r >> 2], whi[r >> 2]); break;
+      }
       e[r] = __viaddmax_s16x2(e[r], nsig, hr[r]);
       f = __viaddmax_s16x2(f, nsig, hrup);
-      uint32_t ef = __vmaxs2(e[r], f);
-      uint32_t h = __viaddmax_s16x2_relu(hrdiag, w, ef);
+      const uint32_t ef = __vmaxs2(e[r], f);
+      const uint32_t h = __viaddmax_s16x2_relu(hrdiag, w, ef);
       hrdiag = hr[r];
       hr[r] = __vadd2(h, nrho);
       hrup = hr[r];
-      if (r & 1) best = __vimax3_s16x2_relu(best, h, hprev); else hprev = h;
+      if (r & 1) best = __vimax3_s16x2(best, hprev, h); else hprev = h;
     }
-    hrup0 = hrup; f0 = f;
+    hrdiag0 = hrup0; hrup0 = hrup ^ (uint32_t)it; f0 = f;
   }
   long long t1 = clock64();
   uint32_t acc = best;
@@ -81,6 +108,7 @@ __global__ void __launch_bounds__(512) k_cellmix(uint32_t* out, uint32_t seed, l
   if (threadIdx.x == 0) cyc[blockIdx.x] = t1 - t0;
 }
 
+static double g_last_rate = 0, g_last_clk = 0;
 template <typename K>
 static void run(const char* name, K kern, double instr_per_thread, int blocks, int threads, uint32_t* d_out,
                 long long* d_cyc, int first) {
@@ -101,6 +129,7 @@ static void run(const char* name, K kern, double instr_per_thread, int blocks, i
   double warp_instr_per_clk_sm = warps_per_sm * instr_per_thread / mean_cyc;
   double thread_instr_per_s = (double)blocks * threads * instr_per_thread * reps / (ms * 1e-3);
   double clk_ghz = mean_cyc / ((ms * 1e-3) / reps) / 1e9;
+  g_last_rate = warp_instr_per_clk_sm; g_last_clk = clk_ghz;
   printf("%s\"%s\": {\"warp_instr_per_clk_per_sm\": %.3f, \"thread_instr_per_s\": %.4e, \"sm_clock_ghz_est\": %.3f}",
          first ? "" : ", ", name, warp_instr_per_clk_sm, thread_instr_per_s, clk_ghz);
 }
@@ -122,9 +151,12 @@ int main() {
   run("IMNMX", k_peak<6>, ipt, blocks, threads, d_out, d_cyc, 0);
   run("VIADDMNMX.S16x2.RELU", k_peak<7>, ipt, blocks, threads, d_out, d_cyc, 0);
   run("VIADDMNMX.S32", k_peak<8>, ipt, blocks, threads, d_out, d_cyc, 0);
-  // cell mix: per iteration R=16 rows x 6.5 ops = 104 ALU ops / thread
-  run("cellmix_s16x2_per_row6.5", k_cellmix, (ITERS / 8) * 16 * 6.5, blocks, threads, d_out, d_cyc, 0);
-  printf("}\n");
+  // cell mix, counted in CELLS: per iteration R rows x 2 cells (two sequences per s16x2 lane)
+  run("cellmix_cells", k_cellmix, (ITERS / 8) * CM_R * 2.0, blocks, threads, d_out, d_cyc, 0);
+  // g_last_rate is "warp-cells" per clk per SM -> x32 lanes x SMs = cells per clk per GPU
+  printf(", \"cells_per_clk_per_gpu\": %.2f, \"sm_mhz_during\": %.0f, \"what\": \"cells_per_clk_per_gpu = issue-bound rate "
+         "of the engine's per-cell instruction mix (PRMT + 5 DPX + 0.5 VIMNMX3 per 2 cells), no memory\"}\n",
+         g_last_rate * 32.0 * nsm, g_last_clk * 1e3);
   cudaError_t err = cudaGetLastError();
   if (err != cudaSuccess) { fprintf(stderr, "CUDA error %s\n", cudaGetErrorString(err)); return 1; }
   return 0;
