@@ -50,6 +50,8 @@ struct sw_handle_s {
   int n_pairs = 0;
   std::vector<int64_t> sorted_len;     // lengths in sorted (descending) order
   std::vector<int32_t> h_pair_ncols;
+  std::vector<int64_t> pair_cols_prefix;  // prefix sums of h_pair_ncols
+  KernelConfig last_cfg{};
   uint16_t* d_cols = nullptr;
   int64_t* d_pair_off = nullptr;
   int32_t* d_pair_ncols = nullptr;
@@ -106,40 +108,89 @@ int grow(sw_handle h, T** p, size_t* cap, size_t bytes, const char* what, cudaSt
 int64_t round_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
 
 // ------------------------------------------------------------------------------------ planning
+ProfLayout make_layout(int off, int G, int R, int m, int A1, int nrep) {
+  ProfLayout L;
+  L.off = off;
+  L.G = G;
+  L.R = R;
+  L.cb = (R % 8 == 0) ? 8 : 4;
+  L.strips = (m + G * R - 1) / (G * R);
+  L.ls = (int)round_up((int64_t)L.strips * G * R, 128);
+  L.nrep = nrep;
+  L.rs = (int)round_up((int64_t)A1 * L.ls, 128) + (nrep > 1 ? (L.cb * G) % 128 : 0);
+  L.bytes = (int)round_up((int64_t)(nrep - 1) * L.rs + (int64_t)A1 * L.ls, 128);
+  return L;
+}
+
 struct Plan {
   KernelConfig cfg;
   int short_passes, long_passes, team_warps;
-  int m_pad, pstride, prof_bytes;
+  ProfLayout lg, lt;   // main kernel blob
+  int prof_bytes;
   // s32 recompute
   KernelConfig rcfg;
   int r_passes, r_team_warps;
+  ProfLayout rl;       // recompute blob (team image only)
+  int r_prof_bytes;
   int grid, rgrid;
 };
 
-int team_warps_for(int passes) {
+int team_warps_for(int passes, int warps) {
   if (passes <= 1) return 1;
-  const int rounds = (passes + kWarps - 1) / kWarps;
+  const int rounds = (passes + warps - 1) / warps;
   return (passes + rounds - 1) / rounds;
 }
 
-// Pick the menu entry minimising the estimated issue cost: padded rows x (1 + per-step
-// overhead / per-step cell work) for each regime, weighted by the regime's residue share.
-int make_plan(sw_handle h, int m, double long_frac, Plan* pl) {
+void main_layouts(const KernelConfig& c, int m, int A1, ProfLayout* lg, ProfLayout* lt, int* bytes) {
+  *lg = make_layout(0, c.G, c.Rs, m, A1, 32 / c.G);
+  if (c.G == 32 && c.Rs == c.Rl) {
+    *lt = *lg;
+    *bytes = lg->bytes;
+  } else {
+    *lt = make_layout(lg->bytes, 32, c.Rl, m, A1, 1);
+    *bytes = lg->bytes + lt->bytes;
+  }
+}
+
+constexpr int kMaxProfileSmem = 220 * 1024;
+
+// Workload summary of one regime split (from the sorted, paired layout).
+struct Split {
+  int n_long = 0, n_short = 0;          // pairs
+  int64_t long_cols = 0, short_cols = 0;
+  int64_t long_max_cols = 0, short_max_cols = 0;
+};
+
+// Pick the menu entry with the smallest estimated time: the larger of
+//  * throughput: warp-steps x ALU instructions per step / the SM array's measured issue rate
+//    (group steps = sum over short pairs of (n' + G - 1) x strips / pairs per warp; team
+//    steps = sum over long pairs of (n' + 31) x strips), and
+//  * the critical path of the longest item (long: its strips split over the team's warps;
+//    short: one group), at the issue rate one warp gets while sharing its scheduler.
+int make_plan(sw_handle h, int m, const Split& sp, Plan* pl) {
   const int A1 = h->A + 1;
+  const double kGpuIssue = 2.7 * h->num_sms;  // ALU warp-instructions per clock, whole GPU
+  const double kWarpIssue = 0.2;              // one warp's share of its scheduler
   double best = 1e300;
   int best_i = -1;
   for (int i = 0; i < menu_size(); ++i) {
     const KernelConfig c = menu_entry(i);
     if (c.lane != 0) continue;
-    const int rs = c.G * c.Rs, rl = 32 * c.Rl;
-    const int ps = (m + rs - 1) / rs, plong = (m + rl - 1) / rl;
-    const int rpass = (m + 32 * 16 - 1) / (32 * 16);
-    const int m_pad = std::max({ps * rs, plong * rl, rpass * 32 * 16});
-    const int64_t bytes = (int64_t)A1 * round_up(m_pad, 16);
-    if (bytes > 200 * 1024) continue;
-    const double cs = (double)ps * rs * (1.0 + 22.0 / (6.5 * c.Rs)) * (1.0 + (c.G - 1) / (ps * 350.0));
-    const double cl = (double)plong * rl * (1.0 + 22.0 / (6.5 * c.Rl));
-    const double cost = cs * (1.0 - long_frac) + cl * long_frac;
+    ProfLayout lg, lt;
+    int bytes = 0;
+    main_layouts(c, m, A1, &lg, &lt, &bytes);
+    if (bytes > kMaxProfileSmem) continue;
+    // several strips in group mode are only efficient for whole-warp chains: with G < 32 the
+    // strip-boundary row traffic per cell grows by 32 / G and its latency dominates (measured)
+    if (lg.strips > 1 && c.G < 32) continue;
+    const double is = 6.5 * c.Rs + 24.0, il = 6.5 * c.Rl + 40.0;   // ALU instructions per step
+    const int W = team_warps_for(lt.strips, c.threads / 32);
+    const double gsteps = ((double)sp.short_cols + (double)sp.n_short * (c.G - 1)) * lg.strips / (32 / c.G);
+    const double tsteps = ((double)sp.long_cols + 31.0 * sp.n_long) * lt.strips;
+    const double thr = (gsteps * is + tsteps * il) / kGpuIssue;
+    const double tail_l = sp.n_long ? (sp.long_max_cols + 31.0) * ((lt.strips + W - 1) / W) * il / kWarpIssue : 0.0;
+    const double tail_s = sp.n_short ? (sp.short_max_cols + c.G - 1.0) * lg.strips * is / kWarpIssue : 0.0;
+    const double cost = std::max(thr, std::max(tail_l, tail_s));
     if (cost < best) { best = cost; best_i = i; }
   }
   // test hooks: force a menu entry / team size (used by the parity tests to cover every
@@ -151,25 +202,27 @@ int make_plan(sw_handle h, int m, double long_frac, Plan* pl) {
   if (best_i < 0) return fail(h, SW_E_UNSUPPORTED, "query profile does not fit in shared memory (query_len * (alphabet_size + 1) too large)");
   const KernelConfig c = menu_entry(best_i);
   pl->cfg = c;
-  pl->short_passes = (m + c.G * c.Rs - 1) / (c.G * c.Rs);
-  pl->long_passes = (m + 32 * c.Rl - 1) / (32 * c.Rl);
-  pl->team_warps = team_warps_for(pl->long_passes);
+  main_layouts(c, m, A1, &pl->lg, &pl->lt, &pl->prof_bytes);
+  if (pl->prof_bytes > kMaxProfileSmem) return fail(h, SW_E_UNSUPPORTED, "query profile does not fit in shared memory");
+  pl->short_passes = pl->lg.strips;
+  pl->long_passes = pl->lt.strips;
+  pl->team_warps = team_warps_for(pl->long_passes, c.threads / 32);
   if (const char* f = getenv("SW_FORCE_TEAM_WARPS")) {
     const int w = atoi(f);
-    if (w >= 1 && w <= kWarps) pl->team_warps = std::min(w, std::max(1, pl->long_passes));
+    if (w >= 1 && w <= c.threads / 32) pl->team_warps = std::min(w, std::max(1, pl->long_passes));
   }
   pl->rcfg = recompute_config();
-  pl->r_passes = (m + 32 * pl->rcfg.Rl - 1) / (32 * pl->rcfg.Rl);
-  pl->r_team_warps = team_warps_for(pl->r_passes);
-  pl->m_pad = std::max({pl->short_passes * c.G * c.Rs, pl->long_passes * 32 * c.Rl, pl->r_passes * 32 * pl->rcfg.Rl});
-  pl->pstride = (int)round_up(pl->m_pad, 16);
-  pl->prof_bytes = A1 * pl->pstride;
+  pl->rl = make_layout(0, 32, pl->rcfg.Rl, m, A1, 1);
+  pl->r_prof_bytes = pl->rl.bytes;
+  if (pl->r_prof_bytes > kMaxProfileSmem) return fail(h, SW_E_UNSUPPORTED, "query profile does not fit in shared memory");
+  pl->r_passes = pl->rl.strips;
+  pl->r_team_warps = team_warps_for(pl->r_passes, pl->rcfg.threads / 32);
   int bps = 0;
   cudaError_t e = configure_kernel(c, pl->prof_bytes, &bps);
   if (e != cudaSuccess) return cuda_fail(h, e, "configure search kernel");
   if (bps < 1) return fail(h, SW_E_UNSUPPORTED, "search kernel cannot be resident");
   pl->grid = bps * h->num_sms;
-  e = configure_kernel(pl->rcfg, pl->prof_bytes, &bps);
+  e = configure_kernel(pl->rcfg, pl->r_prof_bytes, &bps);
   if (e != cudaSuccess) return cuda_fail(h, e, "configure recompute kernel");
   if (bps < 1) return fail(h, SW_E_UNSUPPORTED, "recompute kernel cannot be resident");
   pl->rgrid = bps * h->num_sms;
@@ -204,37 +257,40 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
       std::lower_bound(h->sorted_len.begin(), h->sorted_len.end(), (int64_t)T, std::greater_equal<int64_t>()) -
       h->sorted_len.begin();
   const int n_long = (int)((n_long_seqs + 1) / 2);
-  int64_t long_cols = 0, all_cols = 0;
-  for (int p = 0; p < h->n_pairs; ++p) {
-    all_cols += h->h_pair_ncols[p];
-    if (p < n_long) long_cols += h->h_pair_ncols[p];
-  }
-  const double long_frac = all_cols ? (double)long_cols / (double)all_cols : 0.0;
+  Split sp;
+  sp.n_long = n_long;
+  sp.n_short = h->n_pairs - n_long;
+  sp.long_cols = h->pair_cols_prefix[n_long];
+  sp.short_cols = h->pair_cols_prefix[h->n_pairs] - sp.long_cols;
+  sp.long_max_cols = n_long ? h->h_pair_ncols[0] : 0;
+  sp.short_max_cols = sp.n_short ? h->h_pair_ncols[n_long] : 0;
   Plan pl;
-  int rc = make_plan(h, m, long_frac, &pl);
+  int rc = make_plan(h, m, sp, &pl);
   if (rc) return rc;
+  h->last_cfg = pl.cfg;
 
   // scratch: profile, overflow list, row buffers
-  rc = grow(h, &s.d_prof, &s.prof_cap, (size_t)pl.prof_bytes, "alloc profile", s.stream);
+  const int r_off = (int)round_up(pl.prof_bytes, 256);
+  rc = grow(h, &s.d_prof, &s.prof_cap, (size_t)(r_off + pl.r_prof_bytes), "alloc profile", s.stream);
   if (rc) return rc;
   size_t ovf_bytes = (size_t)std::max<int64_t>(h->n_seqs, 1) * sizeof(int32_t);
   size_t ovf_cap = (size_t)s.ovf_cap * sizeof(int32_t);
   rc = grow(h, &s.d_ovf_list, &ovf_cap, ovf_bytes, "alloc overflow list", s.stream);
   if (rc) return rc;
   s.ovf_cap = (int64_t)(ovf_cap / sizeof(int32_t));
-  const int64_t max_cols_all = h->n_pairs ? h->h_pair_ncols[0] : 0;
-  const int64_t max_cols_short = (n_long < h->n_pairs) ? h->h_pair_ncols[n_long] : 0;
+  const int64_t max_cols_all = h->n_pairs ? h->h_pair_ncols[0] + kPadCols : 0;
+  const int64_t max_cols_short = (n_long < h->n_pairs) ? h->h_pair_ncols[n_long] + kPadCols : 0;
   const int G = pl.cfg.G;
   size_t rbg = 0;
   if (pl.short_passes > 1 && max_cols_short > 0)
-    rbg = (size_t)pl.grid * kWarps * (32 / G) * max_cols_short * sizeof(uint2);
+    rbg = (size_t)pl.grid * (pl.cfg.threads / 32) * (32 / G) * max_cols_short * sizeof(uint2);
   size_t rbt = 0;
   if (pl.long_passes > 1 && n_long > 0) {
-    const int nteams = kWarps / pl.team_warps;
-    rbt = (size_t)pl.grid * nteams * (pl.team_warps + 1) * h->h_pair_ncols[0] * sizeof(uint2);
+    const int nteams = (pl.cfg.threads / 32) / pl.team_warps;
+    rbt = (size_t)pl.grid * nteams * (pl.team_warps + 1) * max_cols_all * sizeof(uint2);
   }
   if (pl.r_passes > 1) {
-    const int nteams = kWarps / pl.r_team_warps;
+    const int nteams = (pl.rcfg.threads / 32) / pl.r_team_warps;
     rbt = std::max(rbt, (size_t)pl.rgrid * nteams * (pl.r_team_warps + 1) * max_cols_all * sizeof(uint2));
   }
   rc = grow(h, &s.d_rb_group, &s.rb_group_cap, rbg, "alloc group row buffers", s.stream);
@@ -245,12 +301,15 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   cudaStream_t st = s.stream;
   SW_CUDA(h, cudaMemsetAsync(s.d_work, 0, 4 * sizeof(int32_t), st));
   SW_CUDA(h, cudaMemsetAsync(s.d_ovf_count, 0, sizeof(int32_t), st));
-  SW_CUDA(h, launch_profile(s.d_prof, d_q, m, h->d_matrix, h->A, h->rho, pl.pstride, st));
+  SW_CUDA(h, launch_profile(s.d_prof, pl.lg, d_q, m, h->d_matrix, h->A, h->rho, st));
+  if (pl.lt.off != pl.lg.off) SW_CUDA(h, launch_profile(s.d_prof, pl.lt, d_q, m, h->d_matrix, h->A, h->rho, st));
+  SW_CUDA(h, launch_profile(s.d_prof + r_off, pl.rl, d_q, m, h->d_matrix, h->A, h->rho, st));
 
   SearchParams p{};
   p.prof = s.d_prof;
-  p.pstride = pl.pstride;
   p.prof_bytes = pl.prof_bytes;
+  p.lg = pl.lg;
+  p.lt = pl.lt;
   p.pad_letter = h->A;
   p.rho = h->rho;
   p.sigma = h->sigma;
@@ -281,18 +340,22 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
 
   // exact 32-bit recompute of sequences whose 16-bit best reached 32767 - max_w
   SearchParams r = p;
+  r.prof = s.d_prof + r_off;
+  r.prof_bytes = pl.r_prof_bytes;
+  r.lg = pl.rl;
+  r.lt = pl.rl;
   r.item_list = s.d_ovf_list;
   r.item_count = s.d_ovf_count;
   r.work = s.d_work + 2;
   r.long_passes = pl.r_passes;
   r.team_warps = pl.r_team_warps;
-  SW_CUDA(h, launch_search(pl.rcfg, r, pl.rgrid, pl.prof_bytes, st));
+  SW_CUDA(h, launch_search(pl.rcfg, r, pl.rgrid, pl.r_prof_bytes, st));
   SW_CUDA(h, cudaEventRecord(ev[2], st));
   SW_CUDA(h, cudaMemcpyAsync(h_ovf, s.d_ovf_count, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
 
   h->stat_long += n_long_seqs;
   h->stat_short += h->n_seqs - n_long_seqs;
-  h->stat_launches += 3;
+  h->stat_launches += 4 + (pl.lt.off != pl.lg.off ? 1 : 0);
   return SW_OK;
 }
 
@@ -438,9 +501,11 @@ int sw_load_db(sw_handle h, const uint8_t* residues, int64_t total_residues, con
     const int64_t hi = (2 * p + 1 < num_seqs) ? h->sorted_len[2 * p + 1] : 0;
     const int64_t nc = round_up(std::max<int64_t>({lo, hi, (int64_t)kMinCols}), kColAlign);
     h->h_pair_ncols[p] = (int32_t)nc;
-    pair_off[p + 1] = pair_off[p] + nc;
+    pair_off[p + 1] = pair_off[p] + nc + kPadCols;
   }
   const int64_t total_cols = pair_off[n_pairs];
+  h->pair_cols_prefix.assign((size_t)n_pairs + 1, 0);
+  for (int p = 0; p < n_pairs; ++p) h->pair_cols_prefix[p + 1] = h->pair_cols_prefix[p] + h->h_pair_ncols[p];
   std::vector<uint16_t> cols((size_t)std::max<int64_t>(total_cols, 1));
   const uint16_t pad = (uint16_t)h->A;
   for (int p = 0; p < n_pairs; ++p) {
@@ -453,7 +518,7 @@ int sw_load_db(sw_handle h, const uint8_t* residues, int64_t total_residues, con
     const int64_t s1 = has1 ? perm[2 * p + 1] : 0;
     const int64_t l1 = has1 ? len[s1] : 0;
     const uint8_t* r1 = (has1 && residues) ? residues + offsets[s1] : nullptr;
-    for (int64_t j = 0; j < nc; ++j) {
+    for (int64_t j = 0; j < nc + kPadCols; ++j) {
       const uint16_t a = j < l0 ? r0[j] : pad;
       const uint16_t b = j < l1 ? r1[j] : pad;
       dst[j] = (uint16_t)(a | (b << 8));

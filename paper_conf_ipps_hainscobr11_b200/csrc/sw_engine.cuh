@@ -29,6 +29,7 @@
 //     with 32-bit lanes (LaneS32) by the same engine.
 #pragma once
 #include <cstdint>
+#include <type_traits>
 #include <cuda_runtime.h>
 
 #include "sw_internal.h"
@@ -64,6 +65,10 @@ struct LaneS16x2 {
   static __device__ __forceinline__ uint32_t max3(uint32_t a, uint32_t b, uint32_t c) {
     return __vimax3_s16x2(a, b, c);
   }
+  // max(t, e, f, 0)
+  static __device__ __forceinline__ uint32_t hmax(uint32_t t, uint32_t e, uint32_t f) {
+    return __vimax3_s16x2_relu(t, e, f);
+  }
   // substitution value of profile row k (of a 4-row int8 word) for both sequences,
   // sign-extended to two s16 halves with one PRMT
   template <int K>
@@ -85,6 +90,9 @@ struct LaneS32 {
   static __device__ __forceinline__ uint32_t add(uint32_t a, uint32_t b) { return a + b; }
   static __device__ __forceinline__ uint32_t max3(uint32_t a, uint32_t b, uint32_t c) {
     return (uint32_t)__vimax3_s32((int)a, (int)b, (int)c);
+  }
+  static __device__ __forceinline__ uint32_t hmax(uint32_t t, uint32_t e, uint32_t f) {
+    return (uint32_t)__vimax3_s32_relu((int)t, (int)e, (int)f);
   }
   template <int K>
   static __device__ __forceinline__ uint32_t subst(uint32_t wlo, uint32_t) {
@@ -141,25 +149,37 @@ __device__ __forceinline__ void team_bar(int team, int W) {
   }
 }
 
-// R bytes of one profile letter row -> R/4 words (4 query rows per word, §III-B
-// "stores the similarity scores of four symbols in a single variable")
-template <int R>
+// R rows of one letter for one lane -> R/4 words (4 query rows per word, §III-B
+// "stores the similarity scores of four symbols in a single variable").  The lane's rows are
+// R/CB chunks of CB bytes, STRIDE bytes apart (ProfLayout).
+template <int R, int CB, int STRIDE>
 __device__ __forceinline__ void load_prof(uint32_t (&w)[R / 4], const uint8_t* p) {
-  if constexpr (R % 16 == 0) {
+  static_assert(R % CB == 0, "R must be a multiple of the chunk size");
+  if constexpr (CB == 8) {
 #pragma unroll
-    for (int i = 0; i < R / 16; ++i) {
-      const uint4 v = reinterpret_cast<const uint4*>(p)[i];
-      w[4 * i + 0] = v.x; w[4 * i + 1] = v.y; w[4 * i + 2] = v.z; w[4 * i + 3] = v.w;
-    }
-  } else if constexpr (R % 8 == 0) {
-#pragma unroll
-    for (int i = 0; i < R / 8; ++i) {
-      const uint2 v = reinterpret_cast<const uint2*>(p)[i];
-      w[2 * i + 0] = v.x; w[2 * i + 1] = v.y;
+    for (int k = 0; k < R / 8; ++k) {
+      const uint2 v = *reinterpret_cast<const uint2*>(p + k * STRIDE);
+      w[2 * k + 0] = v.x; w[2 * k + 1] = v.y;
     }
   } else {
 #pragma unroll
-    for (int i = 0; i < R / 4; ++i) w[i] = reinterpret_cast<const uint32_t*>(p)[i];
+    for (int k = 0; k < R / 4; ++k) w[k] = *reinterpret_cast<const uint32_t*>(p + k * STRIDE);
+  }
+}
+
+template <int R>
+__host__ __device__ constexpr int chunk_bytes() { return (R % 8 == 0) ? 8 : 4; }
+
+// substitution value (w + rho) of row r of the lane's window, packed per Lane
+template <class L, int R>
+__device__ __forceinline__ uint32_t subst_row(const uint32_t (&wlo)[R / 4], const uint32_t (&whi)[R / 4], int r) {
+  const uint32_t a = wlo[r >> 2];
+  const uint32_t b = (L::kSeqs == 2) ? whi[r >> 2] : 0u;
+  switch (r & 3) {
+    case 0: return L::template subst<0>(a, b);
+    case 1: return L::template subst<1>(a, b);
+    case 2: return L::template subst<2>(a, b);
+    default: return L::template subst<3>(a, b);
   }
 }
 
@@ -168,119 +188,140 @@ __device__ __forceinline__ uint32_t pass_tag(int pass, int cols_done) {
 }
 
 struct ChainConst {
-  const uint8_t* sprof;   // shared-memory profile
-  int pstride;
   int rho, sigma;
   uint32_t padpair;       // residue pair of two pad letters
 };
 
-// One chain of GC lanes sweeping `steps` pipeline steps over its passes (see file header).
-// Returns this lane's running best (packed per Lane).
-template <class L, int GC, int R, bool TEAM>
-__device__ __forceinline__ uint32_t run_chain(const ChainConst& c, const uint16_t* __restrict__ cols, int ncols,
-                                              int half, int steps, int pass0, int pstep, int npass,
-                                              int passes_total, uint2* __restrict__ rb, int64_t rb_cols,
-                                              int rb_nslot, uint32_t* prog) {
-  static_assert(R % 4 == 0 && R % 2 == 0, "R must be a multiple of 4");
+// One strip pass of a chain of GC lanes over the columns of one database pair (see the file
+// header).  Lane l owns rows [(P*GC + l)*R, +R) of the query and processes column j at step
+// j + l.  All lanes start the pass in the neutral state (H = 0 -> hr = -rho, E = -inf -> -rho
+// by reading c4); a lane still in its pipeline fill sees neutral inputs and pad letters, which
+// keep it exactly neutral, so no per-lane reset is needed inside the step loop.
+// Returns max(best, this lane's H maxima) (packed per Lane).
+template <class L, int GC, int R, bool TEAM, bool PP>
+__device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t* prow, int ls,
+                                             const uint16_t* __restrict__ cols, int ncols,
+                                             int half, int steps, int P, int passes_total,
+                                             const uint2* __restrict__ rb_in, uint2* __restrict__ rb_out,
+                                             const uint32_t* prog_in, uint32_t* prog_out, uint32_t best) {
+  static_assert(R % 4 == 0, "R must be a multiple of 4");
   const int lane = threadIdx.x & 31;
   const int gl = lane & (GC - 1);
   const uint32_t nrho = L::splat(-c.rho);
   const uint32_t nsig = L::splat(-c.sigma);
   const int hshift = 8 * half;
+  constexpr int CB = chunk_bytes<R>();
+  const bool store_out = (gl == GC - 1) && (P < passes_total - 1);
+  const bool from_prev = P > 0;
 
-  uint32_t hr[R], e[R];
+  // PP: the unrolled step loop ping-pongs between two register arrays (H - rho of the left
+  // column / of this column) so the allocator needs fewer copies (§III-A: keep
+  // the tile in registers); without PP one array is updated in place (fewer registers, more
+  // resident warps, some register moves on the FMA pipe).
+  uint32_t hrA[R], hrB[PP ? R : 1], e[R];
 #pragma unroll
-  for (int r = 0; r < R; ++r) { hr[r] = nrho; e[r] = nrho; }
-  uint32_t best = 0, hrdiag0 = nrho;
-  uint32_t y_hr = nrho, y_f = nrho, y_res = c.padpair;
-  int col = -gl, k = 0, P = pass0;
-  const uint8_t* prow = c.sprof;  // row window of this lane in the profile (set at column 0)
+  for (int r = 0; r < R; ++r) { hrA[r] = nrho; e[r] = nrho; }
+  if constexpr (PP) {
+#pragma unroll
+    for (int r = 0; r < R; ++r) hrB[r] = nrho;
+  }
+  // neutral state: H = 0 on the row above / left column, E = F = -rho (<= 0, reading c4)
+  uint32_t hrdiag0 = nrho;
+  uint32_t y_hr = 0, y_f = 0, y_res = c.padpair;   // (H, F + rho) of this lane's bottom row
+  int col = -gl;
 
-  // lane 0 of the chain streams residues and the previous strip's bottom row, one step ahead
-  uint32_t in_res = c.padpair, in_hr = nrho, in_f = nrho;
-  auto fetch = [&](int fk, int fcol, int fP) {
-    in_res = c.padpair; in_hr = nrho; in_f = nrho;
-    if (fk < npass) {
-      in_res = cols[fcol];
-      if (fP > 0) {
-        const int slot = TEAM ? ((fP - 1) % rb_nslot) : 0;
-        if (TEAM && (fcol & 7) == 0) {
-          const uint32_t need = pass_tag(fP - 1, fcol + 8);
-          while (ld_acquire_smem(prog + slot) < need) __nanosleep(20);
+  // Lane 0 streams residues and the previous strip's bottom row through a 4-deep register
+  // ring: the loads for column j + 4 are issued while column j is computed, so L2 latency is
+  // hidden behind four steps of DP work.  Every pair is stored with kPadCols trailing pad
+  // columns, so the stream runs branch-free past the last column (clamped to the last pad
+  // column): the lanes then compute the DP of the sequence extended by pad letters, whose
+  // optimum is the same (a pad column only adds -128 substitutions or gaps, so truncating an
+  // alignment at the last real column never lowers its score).  The previous strip's last
+  // lane wrote columns 0 .. steps - GC; later columns reuse the last one (bounded, legitimate
+  // DP values of the extended matrix).
+  const int cmax = ncols + kPadCols - 1;
+  const int rlast = steps - GC;
+  uint32_t ring_res[4], ring_h[4], ring_f[4];   // top boundary: H[0][j] = 0, F[0][j] + rho <= 0
+#pragma unroll
+  for (int k = 0; k < 4; ++k) { ring_res[k] = c.padpair; ring_h[k] = 0; ring_f[k] = 0; }
+  uint32_t known = 0;   // team mode: last progress value seen for strip P - 1
+  auto fetch = [&](int k, int fcol) {
+    ring_res[k] = cols[min(fcol, cmax)];
+    if (from_prev) {
+      const int rc = min(fcol, rlast);
+      if constexpr (TEAM) {
+        const uint32_t need = pass_tag(P - 1, rc + 1);
+        if (known < need) {
+          while ((known = ld_acquire_smem(prog_in)) < need) __nanosleep(32);
         }
-        const uint2 v = rb[slot * rb_cols + fcol];
-        in_hr = v.x; in_f = v.y;
       }
+      const uint2 v = rb_in[rc];
+      ring_h[k] = v.x; ring_f[k] = v.y;
     }
   };
-  if (gl == 0) fetch(0, 0, pass0);
+  if (gl == 0) {
+#pragma unroll
+    for (int k = 0; k < 4; ++k) fetch(k, k);
+  }
 
-  for (int s = 0; s < steps; ++s) {
+  auto step = [&](auto kc, uint32_t* hin, uint32_t* hout) {
+    constexpr int K = decltype(kc)::value;
     uint32_t x_hr = __shfl_up_sync(SWB_FULL, y_hr, 1, GC);
     uint32_t x_f = __shfl_up_sync(SWB_FULL, y_f, 1, GC);
     uint32_t x_res = __shfl_up_sync(SWB_FULL, y_res, 1, GC);
-    if (gl == 0) { x_hr = in_hr; x_f = in_f; x_res = in_res; }
-    if (col == 0) {
-      // first column of a strip: H[i][0] = 0 (hr = -rho), E[i][0] = -inf (reading c4: any
-      // value <= 0 gives the same H; -rho is used), diagonal of row 0 is H[r0-1][0] = 0.
-#pragma unroll
-      for (int r = 0; r < R; ++r) { hr[r] = nrho; e[r] = nrho; }
-      hrdiag0 = nrho;
-      // past the last strip the lane only sees pad columns: keep the window in bounds
-      prow = c.sprof + (k < npass ? (P * GC + gl) * R : 0);
-    }
+    if (gl == 0) { x_hr = ring_h[K]; x_f = ring_f[K]; x_res = ring_res[K]; }
     // query-profile words for the two letters of this column
     uint32_t wlo[R / 4], whi[R / 4];
     {
       const int alo = (x_res >> hshift) & 0xff;
-      load_prof<R>(wlo, prow + alo * c.pstride);
+      load_prof<R, CB, GC * CB>(wlo, prow + alo * ls);
       if constexpr (L::kSeqs == 2) {
         const int ahi = x_res >> 8;
-        load_prof<R>(whi, prow + ahi * c.pstride);
+        load_prof<R, CB, GC * CB>(whi, prow + ahi * ls);
       }
     }
-    uint32_t hrup = x_hr, f = x_f, hrdiag = hrdiag0, hprev = 0;
+    if (gl == 0) fetch(K, col + 4);
+    // Vertical values travel as (H, F + rho) so that the F -> H -> F chain down the rows is
+    // two fused DPX ops per row: Fs = F + rho = max(Fs[i-1] - sigma, H[i-1]) and
+    // H = max(Fs - rho, u) with u = max(H[i-1][j-1] + w, E, 0) off the chain.
+    uint32_t hup = x_hr, fs = x_f, hprev = 0;
+    uint32_t hrdiag = hrdiag0;
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-      uint32_t wv;
-      const uint32_t a = wlo[r >> 2];
-      const uint32_t b = (L::kSeqs == 2) ? whi[r >> 2] : 0u;
-      switch (r & 3) {
-        case 0: wv = L::template subst<0>(a, b); break;
-        case 1: wv = L::template subst<1>(a, b); break;
-        case 2: wv = L::template subst<2>(a, b); break;
-        default: wv = L::template subst<3>(a, b); break;
-      }
-      e[r] = L::gap(e[r], nsig, hr[r]);          // E[i][j] = max(E[i][j-1] - sigma, H[i][j-1] - rho)
-      f = L::gap(f, nsig, hrup);                 // F[i][j] = max(F[i-1][j] - sigma, H[i-1][j] - rho)
-      const uint32_t ef = L::max2(e[r], f);
-      const uint32_t h = L::hcell(hrdiag, wv, ef);  // max(H[i-1][j-1] + w, E, F, 0)
-      hrdiag = hr[r];
-      hr[r] = L::add(h, nrho);                   // H - rho
-      hrup = hr[r];
+      e[r] = L::gap(e[r], nsig, hin[r]);                              // E = max(E[j-1] - sigma, H[j-1] - rho)
+      const uint32_t u = L::hcell(hrdiag, subst_row<L, R>(wlo, whi, r), e[r]);  // max(H[i-1][j-1] + w, E, 0)
+      fs = L::gap(fs, nsig, hup);                                     // F + rho = max(F[i-1] + rho - sigma, H[i-1])
+      const uint32_t h = L::gap(fs, nrho, u);                         // H = max(F, u)
+      hrdiag = hin[r];
+      hout[r] = L::add(h, nrho);                                      // H - rho (left value of the next column)
+      hup = h;
       if (r & 1) best = L::max3(best, hprev, h); else hprev = h;
     }
-    hrdiag0 = x_hr;
-    y_hr = hrup; y_f = f; y_res = x_res;
-
-    // last lane: save the strip's bottom row for the next strip (not after the last strip)
-    if (gl == GC - 1 && col >= 0 && k < npass && P < passes_total - 1) {
-      const int slot = TEAM ? (P % rb_nslot) : 0;
-      rb[slot * rb_cols + col] = make_uint2(y_hr, y_f);
-      if (TEAM && ((col & 7) == 7 || col == ncols - 1)) {
-        __threadfence_block();
-        st_release_smem(prog + slot, pass_tag(P, col + 1));
-      }
-    }
-    // lane 0: prefetch the next step's inputs
-    if (gl == 0) {
-      int nk = k, ncol = col + 1, nP = P;
-      if (ncol == ncols) { ncol = 0; ++nk; nP += pstep; }
-      fetch(nk, ncol, nP);
+    hrdiag0 = L::add(x_hr, nrho);
+    y_hr = hup; y_f = fs; y_res = x_res;
+    // last lane: save the strip's bottom row for the next strip (not after the last strip);
+    // fill steps write neutral values that the real column overwrites later.  Team mode
+    // publishes progress every 16 columns (release: the row-buffer stores are visible first).
+    if (store_out) {
+      rb_out[max(col, 0)] = make_uint2(y_hr, y_f);
+      if (TEAM && col >= 0 && ((col & 15) == 15 || col == rlast)) st_release_smem(prog_out, pass_tag(P, col + 1));
     }
     ++col;
-    if (col == ncols) { col = 0; ++k; P += pstep; }
-    if (!TEAM) __syncwarp();
+  };
+
+  // steps is a multiple of 4 (<= ncols + kPadCols); extra steps only see pad columns
+  for (int s = 0; s < steps; s += 4) {
+    if constexpr (PP) {
+      step(std::integral_constant<int, 0>{}, hrA, hrB);
+      step(std::integral_constant<int, 1>{}, hrB, hrA);
+      step(std::integral_constant<int, 2>{}, hrA, hrB);
+      step(std::integral_constant<int, 3>{}, hrB, hrA);
+    } else {
+      step(std::integral_constant<int, 0>{}, hrA, hrA);
+      step(std::integral_constant<int, 1>{}, hrA, hrA);
+      step(std::integral_constant<int, 2>{}, hrA, hrA);
+      step(std::integral_constant<int, 3>{}, hrA, hrA);
+    }
   }
   return best;
 }
@@ -302,13 +343,17 @@ __device__ __forceinline__ void emit(const SearchParams& p, uint32_t b, int pair
   }
 }
 
-template <class L, int G, int Rs, int Rl>
-__global__ void __launch_bounds__(kThreads, 1) k_search(const SearchParams p) {
+template <class L, int G, int Rs, int Rl, int NT, bool PP>
+__global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
+  constexpr int kWarps = NT / 32;
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ __align__(8) uint64_t mbar;
   __shared__ uint32_t sprog[2 * kWarps];
   __shared__ uint32_t sred[kWarps];
   __shared__ int32_t sitem[kWarps];
+
+  // the 32-bit recompute launch exits at once when no sequence was flagged
+  if (p.item_list != nullptr && *p.item_count == 0) return;
 
   // ---- stage the query profile in shared memory with TMA bulk copies (§III-B:
   //      the profile lives in texture memory there; on sm_100a it is smem-resident)
@@ -328,8 +373,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_search(const SearchParams p) {
   mbar_wait(&mbar, 0);
 
   ChainConst c;
-  c.sprof = smem;
-  c.pstride = p.pstride;
   c.rho = p.rho;
   c.sigma = p.sigma;
   c.padpair = (uint32_t)p.pad_letter | ((uint32_t)p.pad_letter << 8);
@@ -366,10 +409,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_search(const SearchParams p) {
         // P + W before all its lanes finished strip P: its lane 0 may wait for strip P + W - 1,
         // which transitively needs the tail of strip P (deadlock for short rows otherwise).
         uint32_t b = 0;
+        const int tsteps = (ncols + 31 + 3) & ~3;
         for (int P = wt; P < p.long_passes; P += W) {
-          const uint32_t bp = run_chain<L, 32, Rl, true>(c, cp, ncols, half, ncols + 31, P, W, 1, p.long_passes,
-                                                         rb, p.rb_team_cols, W + 1, prog);
-          b = L::max2(b, bp);
+          const int si = (P + W) % (W + 1), so = P % (W + 1);   // slot of strip P-1 / strip P
+          constexpr int CBl = chunk_bytes<Rl>();
+          const uint8_t* prow = smem + p.lt.off + (P * (Rl / CBl) * 32 + lane) * CBl;
+          b = run_pass<L, 32, Rl, true, PP>(c, prow, p.lt.ls, cp, ncols, half, tsteps, P, p.long_passes,
+                                        rb + (int64_t)si * p.rb_team_cols, rb + (int64_t)so * p.rb_team_cols,
+                                        prog + si, prog + so, b);
         }
 #pragma unroll
         for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
@@ -398,11 +445,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_search(const SearchParams p) {
       const int pair = p.n_long + base + gi;
       const int ncols = valid ? p.pair_ncols[pair] : 0;
       const uint16_t* cp = p.cols + (valid ? p.pair_off[pair] : 0);
-      const int npass = valid ? p.short_passes : 0;
-      const int steps = (int)__reduce_max_sync(SWB_FULL, (unsigned)(npass * ncols)) + G - 1;
+      const int steps = ((int)__reduce_max_sync(SWB_FULL, (unsigned)ncols) + G - 1 + 3) & ~3;
       uint2* rb = p.rb_group + ((int64_t)(blockIdx.x * kWarps + warp) * GPW + gi) * p.rb_group_cols;
-      uint32_t b = run_chain<L, G, Rs, false>(c, cp, ncols, 0, steps, 0, 1, npass, p.short_passes, rb,
-                                              p.rb_group_cols, 1, nullptr);
+      uint32_t b = 0;
+      for (int P = 0; P < p.short_passes; ++P) {
+        constexpr int CBs = chunk_bytes<Rs>();
+        const uint8_t* prow = smem + p.lg.off + gi * p.lg.rs + (P * (Rs / CBs) * G + gl) * CBs;
+        b = run_pass<L, G, Rs, false, PP>(c, prow, p.lg.ls, cp, ncols, 0, steps, P, p.short_passes, rb, rb, nullptr,
+                                      nullptr, b);
+        __syncwarp();   // strip P's bottom row (written by lane G-1) is read by lane 0 in strip P+1
+      }
 #pragma unroll
       for (int o = G / 2; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
       if (gl == 0 && valid) emit<L>(p, b, pair, 0);
@@ -410,18 +462,18 @@ __global__ void __launch_bounds__(kThreads, 1) k_search(const SearchParams p) {
   }
 }
 
-template <class L, int G, int Rs, int Rl>
+template <class L, int G, int Rs, int Rl, int NT, bool PP>
 cudaError_t launch_search_t(const SearchParams& p, int grid, int smem_bytes, cudaStream_t st) {
-  k_search<L, G, Rs, Rl><<<grid, kThreads, smem_bytes, st>>>(p);
+  k_search<L, G, Rs, Rl, NT, PP><<<grid, NT, smem_bytes, st>>>(p);
   return cudaGetLastError();
 }
 
-template <class L, int G, int Rs, int Rl>
+template <class L, int G, int Rs, int Rl, int NT, bool PP>
 cudaError_t configure_t(int smem_bytes, int* blocks_per_sm) {
-  cudaError_t e = cudaFuncSetAttribute(k_search<L, G, Rs, Rl>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       smem_bytes);
+  cudaError_t e = cudaFuncSetAttribute(k_search<L, G, Rs, Rl, NT, PP>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search<L, G, Rs, Rl>, kThreads,
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search<L, G, Rs, Rl, NT, PP>, NT,
                                                        smem_bytes);
 }
 

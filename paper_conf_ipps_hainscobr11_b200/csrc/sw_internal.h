@@ -6,24 +6,46 @@
 
 namespace swb {
 
-constexpr int kThreads = 512;            // threads per CTA (16 warps)
-constexpr int kWarps = kThreads / 32;
+constexpr int kMaxWarps = 16;            // at most 512 threads per CTA
 constexpr int kMinCols = 48;             // every pair is padded to >= 48 columns (>= G + 16)
 constexpr int kColAlign = 8;             // pair column counts are multiples of 8 (16 bytes)
+constexpr int kPadCols = 32;             // trailing pad columns stored after every pair
 constexpr int kPadValue = -128;          // profile value of pad letters / pad query rows
+
+// Bank-conflict-free shared-memory image of the query profile for chains of G lanes with R
+// rows per lane.  Query row i lives in strip P = i / (G*R),
+// lane gl = (i % (G*R)) / R, row r = i % R, chunk k = r / cb (cb = 4 or 8 rows = bytes):
+//   byte(rep, a, i) = off + rep*rs + a*ls + ((P*(R/cb) + k)*G + gl)*cb + r % cb
+// so at a fixed (strip, chunk) the G lanes of a chain read consecutive cb-byte words of
+// their own letter row: the letter term a*ls is a multiple of 128 B (32 banks) and drops
+// out of the bank index, and the 32/G replicas (one per chain of a warp) are shifted by
+// cb*G bytes, so any mix of letters across the warp is conflict-free.
+struct ProfLayout {
+  int off;     // byte offset of the image in the staged blob
+  int G;       // lanes per chain (32 for team mode)
+  int R;       // rows per lane
+  int cb;      // chunk bytes
+  int strips;  // strips covered (strips * G * R >= m)
+  int ls;      // letter stride, multiple of 128
+  int rs;      // replica stride, == cb * G (mod 128)
+  int nrep;    // replicas (32 / G for group mode, 1 for team mode)
+  int bytes;   // nrep * rs
+};
 
 // One persistent search launch for one query.
 struct SearchParams {
-  // query profile P[a][i] = w(q_i, a) + rho as int8 (a < A), row A = pad; i < m_pad
-  const uint8_t* prof;       // global, (A + 1) * pstride bytes
-  int pstride;               // bytes per letter row (multiple of 16, >= m_pad)
-  int prof_bytes;            // (A + 1) * pstride
+  // query profile (w(q_i, a) + rho as int8, -128 for pad letters / rows), staged as one blob
+  const uint8_t* prof;       // global blob: group image then (if different) team image
+  int prof_bytes;            // blob size (multiple of 16)
+  ProfLayout lg;             // group-mode image
+  ProfLayout lt;             // team-mode image (may alias lg)
   int pad_letter;            // == A
   int rho, sigma, max_w;
   // database, sorted by length descending and paired (2p, 2p+1)
   const uint16_t* cols;      // interleaved columns: cols[pair_off[p] + j] = d_lo[j] | d_hi[j] << 8
   const int64_t* pair_off;   // in u16 units
-  const int32_t* pair_ncols; // padded column count n' (multiple of 8, >= kMinCols)
+  const int32_t* pair_ncols; // padded column count n' (multiple of 8, >= kMinCols); the pair
+                             // occupies n' + kPadCols columns (the tail is pad letters)
   int n_pairs;
   int n_seqs;
   const int32_t* perm;       // sorted position -> caller index
@@ -39,10 +61,10 @@ struct SearchParams {
   // passes over the query: group mode G*R_s rows per pass, team mode 32*R_l rows per pass
   int short_passes;
   int long_passes;
-  int team_warps;            // warps per team (1..kWarps), teams = kWarps / team_warps
+  int team_warps;            // warps per team (1..warps per CTA), teams = warps / team_warps
   // row buffers (strip bottom rows, §III "the bottom row of a strip must
   // be saved for the next pass"), uint2 = (H - rho, F) per column
-  uint2* rb_group; int64_t rb_group_cols;   // per group slot
+  uint2* rb_group; int64_t rb_group_cols;   // per group slot (>= max n' + kPadCols)
   uint2* rb_team;  int64_t rb_team_cols;    // per (team slot, pass mod (team_warps+1))
 };
 
@@ -53,6 +75,8 @@ struct KernelConfig {
   int G;
   int Rs;
   int Rl;
+  int threads;   // CTA size (fewer threads for the register-heavy entries)
+  int pingpong;  // 1: two register arrays for H - rho (see run_pass)
 };
 
 // Launch one search; returns the CUDA error of the launch.
@@ -65,8 +89,8 @@ int menu_size();
 KernelConfig menu_entry(int i);
 KernelConfig recompute_config();
 
-// Profile build: prof[a][i] = (i < m && a < A) ? W[q_i][a] + rho : -128.
-cudaError_t launch_profile(uint8_t* prof, const uint8_t* q, int m, const int8_t* W, int A, int rho,
-                           int pstride, cudaStream_t st);
+// Profile image build: byte(rep, a, i) = (i < m && a < A) ? W[q_i][a] + rho : -128.
+cudaError_t launch_profile(uint8_t* blob, const ProfLayout& L, const uint8_t* q, int m, const int8_t* W, int A,
+                           int rho, cudaStream_t st);
 
 }  // namespace swb
