@@ -364,7 +364,11 @@ int run_batch(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq
   h->stat_long = h->stat_short = h->stat_launches = 0;
   h->stat_nq = nq;
   if (h->n_seqs == 0 || nq == 0) return SW_OK;
-  int rc = ensure_slots(h, std::min(nq, 4));
+  // queries run concurrently on up to SW_STREAMS internal streams (default 4) so that the
+  // tail of one query's persistent launch overlaps the next query
+  int max_streams = 4;
+  if (const char* f = getenv("SW_STREAMS")) max_streams = std::max(1, std::min(16, atoi(f)));
+  int rc = ensure_slots(h, std::min(nq, max_streams));
   if (rc) return rc;
   if (h->h_ovf_cap < nq) {
     if (h->h_ovf) { cudaDeviceSynchronize(); cudaFreeHost(h->h_ovf); }
@@ -379,7 +383,7 @@ int run_batch(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq
     SW_CUDA(h, cudaEventCreate(&e));
     h->ev.push_back(e);
   }
-  const int ns = std::min(nq, 4);
+  const int ns = std::min(nq, max_streams);
   SW_CUDA(h, cudaEventRecord(h->fork, user));
   for (int k = 0; k < ns; ++k) SW_CUDA(h, cudaStreamWaitEvent(h->slots[k].stream, h->fork, 0));
   for (int k = 0; k < nq; ++k) {
