@@ -245,24 +245,27 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
 #pragma unroll
   for (int k = 0; k < 4; ++k) { ring_res[k] = c.padpair; ring_h[k] = 0; ring_f[k] = 0; }
   uint32_t known = 0;   // team mode: last progress value seen for strip P - 1
+  // Every lane of the chain runs the fetch (same addresses as its lane 0: broadcast loads, no
+  // extra traffic) so the warp never diverges; only lane 0 consumes the values.  The team-mode
+  // wait for strip P - 1 is a warp-uniform spin on a shared-memory flag (a divergent spin makes
+  // every later shuffle take the slow diverged path).
   auto fetch = [&](int k, int fcol) {
     ring_res[k] = cols[min(fcol, cmax)];
     if (from_prev) {
       const int rc = min(fcol, rlast);
       if constexpr (TEAM) {
         const uint32_t need = pass_tag(P - 1, rc + 1);
-        if (known < need) {
-          while ((known = ld_acquire_smem(prog_in)) < need) __nanosleep(32);
+        while (known < need) {
+          known = ld_acquire_smem(prog_in);
+          if (known < need) __nanosleep(32);
         }
       }
       const uint2 v = rb_in[rc];
       ring_h[k] = v.x; ring_f[k] = v.y;
     }
   };
-  if (gl == 0) {
 #pragma unroll
-    for (int k = 0; k < 4; ++k) fetch(k, k);
-  }
+  for (int k = 0; k < 4; ++k) fetch(k, k);
 
   auto step = [&](auto kc, uint32_t* hin, uint32_t* hout) {
     constexpr int K = decltype(kc)::value;
@@ -280,7 +283,7 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
         load_prof<R, CB, GC * CB>(whi, prow + ahi * ls);
       }
     }
-    if (gl == 0) fetch(K, col + 4);
+    fetch(K, col + gl + 4);   // lane 0's next column (col + gl is the step index)
     // Vertical values travel as (H, F + rho) so that the F -> H -> F chain down the rows is
     // two fused DPX ops per row: Fs = F + rho = max(Fs[i-1] - sigma, H[i-1]) and
     // H = max(Fs - rho, u) with u = max(H[i-1][j-1] + w, E, 0) off the chain.
