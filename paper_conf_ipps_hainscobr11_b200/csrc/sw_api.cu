@@ -31,6 +31,10 @@ struct QuerySlot {
   size_t rb_group_cap = 0;        // bytes
   uint2* d_rb_team = nullptr;
   size_t rb_team_cap = 0;
+  uint2* d_rb_t = nullptr;        // T-mode strip boundaries
+  size_t rb_t_cap = 0;
+  uint16_t* d_qpair = nullptr;    // T-mode query stream
+  size_t qpair_cap = 0;
   cudaStream_t stream = nullptr;
   cudaEvent_t done = nullptr;
 };
@@ -298,6 +302,34 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   rc = grow(h, &s.d_rb_team, &s.rb_team_cap, rbt, "alloc team row buffers", s.stream);
   if (rc) return rc;
 
+  // Long pairs: T-mode (strips along the database sequence) when the query is short enough
+  // that team mode would have few query strips to spread over warps; team mode otherwise.
+  // SW_LONG_MODE=team|t overrides (tests).
+  bool use_t = n_long > 0 && pl.long_passes <= 2;
+  if (const char* f = getenv("SW_LONG_MODE")) {
+    if (!strcmp(f, "team")) use_t = false;
+    if (!strcmp(f, "t")) use_t = n_long > 0;
+  }
+  const int qcols = (int)round_up(m, 8);
+  const int wp_bytes = (int)round_up((int64_t)(h->A + 1) * 32, 128);
+  const int per_warp = 2 * (h->A + 1) * 32 * kTmodeC;
+  int t_warps = std::min(kTmodeThreads / 32, (kMaxProfileSmem - wp_bytes) / per_warp);
+  if (t_warps < 1) use_t = false;
+  int t_grid = 0;
+  const int t_smem = wp_bytes + t_warps * per_warp;
+  if (use_t) {
+    int bps = 0;
+    cudaError_t e = configure_tmode_kernel(t_smem, &bps);
+    if (e != cudaSuccess) return cuda_fail(h, e, "configure long-sequence kernel");
+    t_grid = std::max(1, bps) * h->num_sms;
+    rc = grow(h, &s.d_qpair, &s.qpair_cap, (size_t)(qcols + kPadCols) * sizeof(uint16_t), "alloc query stream",
+              s.stream);
+    if (rc) return rc;
+    rc = grow(h, &s.d_rb_t, &s.rb_t_cap, (size_t)t_grid * 2 * t_warps * (qcols + kPadCols) * sizeof(uint2),
+              "alloc long-sequence row buffers", s.stream);
+    if (rc) return rc;
+  }
+
   cudaStream_t st = s.stream;
   SW_CUDA(h, cudaMemsetAsync(s.d_work, 0, 4 * sizeof(int32_t), st));
   SW_CUDA(h, cudaMemsetAsync(s.d_ovf_count, 0, sizeof(int32_t), st));
@@ -321,7 +353,8 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   p.n_seqs = (int)h->n_seqs;
   p.perm = h->d_perm;
   p.scores = d_out;
-  p.n_long = n_long;
+  p.n_long = use_t ? 0 : n_long;
+  p.short_begin = n_long;
   p.item_list = nullptr;
   p.item_count = nullptr;
   p.work = s.d_work;
@@ -335,6 +368,40 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   p.rb_team = s.d_rb_team;
   p.rb_team_cols = max_cols_all;
   SW_CUDA(h, cudaEventRecord(ev[0], st));
+  if (use_t) {
+    SW_CUDA(h, launch_qpair(s.d_qpair, d_q, m, qcols + kPadCols, h->A, st));
+    TParams t{};
+    t.matrix = h->d_matrix;
+    t.A = h->A;
+    t.rho = h->rho;
+    t.sigma = h->sigma;
+    t.max_w = h->max_w;
+    t.pad_letter = h->A;
+    t.qpair = s.d_qpair;
+    t.qcols = qcols;
+    t.cols = h->d_cols;
+    t.pair_off = h->d_pair_off;
+    t.pair_ncols = h->d_pair_ncols;
+    t.n_items = n_long;
+    t.n_seqs = (int)h->n_seqs;
+    t.perm = h->d_perm;
+    t.scores = d_out;
+    t.ovf_list = s.d_ovf_list;
+    t.ovf_count = s.d_ovf_count;
+    t.work = s.d_work + 3;
+    t.warps = t_warps;
+    // team size ~ strips of a typical long item (512 database positions per strip), so short
+    // long-items do not leave warps of a team idle: W in {1, 2, 4, 8}, W | t_warps
+    const double avg_strips = (double)sp.long_cols / std::max(1, n_long) / (32.0 * kTmodeC);
+    int W = 1;
+    while (W * 2 <= t_warps && W * 2 <= avg_strips + 0.5 && t_warps % (W * 2) == 0) W *= 2;
+    if (const char* f = getenv("SW_T_TEAM")) W = std::max(1, std::min(t_warps, atoi(f)));
+    while (t_warps % W) --W;
+    t.team_warps = W;
+    t.rb = s.d_rb_t;
+    t.rb_cols = qcols + kPadCols;
+    SW_CUDA(h, launch_tmode(t, t_grid, t_smem, st));
+  }
   SW_CUDA(h, launch_search(pl.cfg, p, pl.grid, pl.prof_bytes, st));
   SW_CUDA(h, cudaEventRecord(ev[1], st));
 
@@ -355,7 +422,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
 
   h->stat_long += n_long_seqs;
   h->stat_short += h->n_seqs - n_long_seqs;
-  h->stat_launches += 4 + (pl.lt.off != pl.lg.off ? 1 : 0);
+  h->stat_launches += 4 + (pl.lt.off != pl.lg.off ? 1 : 0) + (use_t ? 2 : 0);
   return SW_OK;
 }
 
@@ -630,7 +697,7 @@ void sw_destroy(sw_handle h) {
   for (QuerySlot& s : h->slots) {
     if (s.stream) cudaStreamSynchronize(s.stream);
     cudaFree(s.d_prof); cudaFree(s.d_work); cudaFree(s.d_ovf_count); cudaFree(s.d_ovf_list);
-    cudaFree(s.d_rb_group); cudaFree(s.d_rb_team); cudaFree(s.d_query);
+    cudaFree(s.d_rb_group); cudaFree(s.d_rb_team); cudaFree(s.d_query); cudaFree(s.d_rb_t); cudaFree(s.d_qpair);
     if (s.stream) cudaStreamDestroy(s.stream);
     if (s.done) cudaEventDestroy(s.done);
   }

@@ -199,7 +199,7 @@ struct ChainConst {
 // keep it exactly neutral, so no per-lane reset is needed inside the step loop.
 // Returns max(best, this lane's H maxima) (packed per Lane).
 template <class L, int GC, int R, bool TEAM, bool PP>
-__device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t* prow, int ls,
+__device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t* prow, int ls, int hi_off,
                                              const uint16_t* __restrict__ cols, int ncols,
                                              int half, int steps, int P, int passes_total,
                                              const uint2* __restrict__ rb_in, uint2* __restrict__ rb_out,
@@ -280,7 +280,7 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
       load_prof<R, CB, GC * CB>(wlo, prow + alo * ls);
       if constexpr (L::kSeqs == 2) {
         const int ahi = x_res >> 8;
-        load_prof<R, CB, GC * CB>(whi, prow + ahi * ls);
+        load_prof<R, CB, GC * CB>(whi, prow + hi_off + ahi * ls);
       }
     }
     fetch(K, col + gl + 4);   // lane 0's next column (col + gl is the step index)
@@ -417,7 +417,7 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
           const int si = (P + W) % (W + 1), so = P % (W + 1);   // slot of strip P-1 / strip P
           constexpr int CBl = chunk_bytes<Rl>();
           const uint8_t* prow = smem + p.lt.off + (P * (Rl / CBl) * 32 + lane) * CBl;
-          b = run_pass<L, 32, Rl, true, PP>(c, prow, p.lt.ls, cp, ncols, half, tsteps, P, p.long_passes,
+          b = run_pass<L, 32, Rl, true, PP>(c, prow, p.lt.ls, 0, cp, ncols, half, tsteps, P, p.long_passes,
                                         rb + (int64_t)si * p.rb_team_cols, rb + (int64_t)so * p.rb_team_cols,
                                         prog + si, prog + so, b);
         }
@@ -438,14 +438,14 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
   if (p.item_list == nullptr) {
     constexpr int GPW = 32 / G;
     const int gi = lane / G, gl = lane & (G - 1);
-    const int nshort = p.n_pairs - p.n_long;
+    const int nshort = p.n_pairs - p.short_begin;
     for (;;) {
       int base = 0;
       if (lane == 0) base = atomicAdd(&p.work[1], GPW);
       base = __shfl_sync(SWB_FULL, base, 0);
       if (base >= nshort) break;
       const bool valid = base + gi < nshort;
-      const int pair = p.n_long + base + gi;
+      const int pair = p.short_begin + base + gi;
       const int ncols = valid ? p.pair_ncols[pair] : 0;
       const uint16_t* cp = p.cols + (valid ? p.pair_off[pair] : 0);
       const int steps = ((int)__reduce_max_sync(SWB_FULL, (unsigned)ncols) + G - 1 + 3) & ~3;
@@ -454,7 +454,7 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
       for (int P = 0; P < p.short_passes; ++P) {
         constexpr int CBs = chunk_bytes<Rs>();
         const uint8_t* prow = smem + p.lg.off + gi * p.lg.rs + (P * (Rs / CBs) * G + gl) * CBs;
-        b = run_pass<L, G, Rs, false, PP>(c, prow, p.lg.ls, cp, ncols, 0, steps, P, p.short_passes, rb, rb, nullptr,
+        b = run_pass<L, G, Rs, false, PP>(c, prow, p.lg.ls, 0, cp, ncols, 0, steps, P, p.short_passes, rb, rb, nullptr,
                                       nullptr, b);
         __syncwarp();   // strip P's bottom row (written by lane G-1) is read by lane 0 in strip P+1
       }
@@ -463,6 +463,130 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
       if (gl == 0 && valid) emit<L>(p, b, pair, 0);
     }
   }
+}
+
+// ------------------------------------------------------------------------------------ T-mode
+// Long database sequences, transposed.  The paper's
+// intra-task kernel gives one thread block to one long sequence and walks strips of QUERY rows
+// (§III, Fig.4).  Here a CTA team walks strips of the DATABASE sequence instead:
+// lane l of warp w owns C consecutive database positions of strip s = w, w + W, ..., and the
+// chain sweeps the query, so a 35k-residue sequence yields ~70 strips of parallel work for any
+// query length.  Eq.(1) is symmetric under transposition (E <-> F, w(q, d) read as w^T(d, q)),
+// so the same engine (run_pass) computes it; the "profile" of a strip is built by its warp
+// from the substitution matrix (tables P_lo[a][pos] = w(a, d_lo[pos]) + rho and P_hi for the
+// pair's second sequence, chunk-major and conflict-free like the query profile) and the
+// residue stream is the query.  Strip boundaries (the last database position of a strip over
+// all query positions) go through the team row buffers with progress flags, as in team mode.
+template <int C, int NT, bool PP>
+__global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
+  using L = LaneS16x2;
+  constexpr int kWarps = NT / 32;
+  constexpr int CB = chunk_bytes<C>();
+  constexpr int LS = 32 * C;                  // letter stride of one strip table (bytes)
+  extern __shared__ __align__(128) uint8_t smem[];
+  __shared__ uint32_t sprog[2 * kWarps];
+  __shared__ uint32_t sred[kWarps];
+  __shared__ int32_t sitem[kWarps];
+  const int A1 = p.A + 1;
+  const int table_bytes = 2 * A1 * LS;        // lo + hi tables of one warp
+  int8_t* wp = reinterpret_cast<int8_t*>(smem);  // (A+1) x 32: w + rho, pad -> -128
+  uint8_t* tables = smem + ((A1 * 32 + 127) & ~127);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (int t = threadIdx.x; t < A1 * 32; t += blockDim.x) {
+    const int a = t >> 5, d = t & 31;
+    int v = kPadValue;
+    if (a < p.A && d < p.A) v = (int)p.matrix[a * p.A + d] + p.rho;
+    wp[t] = (int8_t)v;
+  }
+  __syncthreads();
+  // teams of W warps (W | warps); several teams per CTA when long items have few strips
+  const int W = p.team_warps;
+  const int nteams = p.warps / W;
+  const int team = warp / W, wt = warp % W;
+  if (team >= nteams) return;
+  ChainConst c;
+  c.rho = p.rho;
+  c.sigma = p.sigma;
+  c.padpair = (uint32_t)p.pad_letter | ((uint32_t)p.pad_letter << 8);
+  uint8_t* tab = tables + warp * table_bytes;
+  const int qsteps = (p.qcols + 31 + 3) & ~3;
+  uint32_t* prog = sprog + team * (W + 1);
+  uint2* rb = p.rb + ((int64_t)blockIdx.x * nteams + team) * (W + 1) * p.rb_cols;
+  for (;;) {
+    team_bar(team, W);
+    if (wt == 0 && lane == 0) {
+      sitem[team] = atomicAdd(p.work, 1);
+      for (int i = 0; i <= W; ++i) prog[i] = 0u;
+    }
+    team_bar(team, W);
+    const int item = sitem[team];
+    if (item >= p.n_items) break;
+    const int ncols = p.pair_ncols[item];
+    const uint16_t* cp = p.cols + p.pair_off[item];
+    const int S = (ncols + LS - 1) / LS;       // strips of the database pair
+    uint32_t b = 0;
+    for (int P = wt; P < S; P += W) {
+      // build this warp's strip tables: position pos = P*LS + lane*C + r
+      __syncwarp();
+      uint32_t dp[C];
+#pragma unroll
+      for (int r = 0; r < C; ++r) {
+        const int pos = P * LS + lane * C + r;
+        dp[r] = pos < ncols ? (uint32_t)cp[pos] : c.padpair;
+      }
+      for (int a = 0; a < A1; ++a) {
+        const int8_t* wrow = wp + a * 32;
+#pragma unroll
+        for (int k = 0; k < C / 4; ++k) {
+          uint32_t lo = 0, hi = 0;
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            const uint32_t d = dp[4 * k + j];
+            lo |= (uint32_t)(uint8_t)wrow[d & 0xff] << (8 * j);
+            hi |= (uint32_t)(uint8_t)wrow[d >> 8] << (8 * j);
+          }
+          const int r0 = 4 * k;
+          const int off = a * LS + ((r0 / CB) * 32 + lane) * CB + (r0 % CB);
+          *reinterpret_cast<uint32_t*>(tab + off) = lo;
+          *reinterpret_cast<uint32_t*>(tab + A1 * LS + off) = hi;
+        }
+      }
+      __syncwarp();
+      const int si = (P + W) % (W + 1), so = P % (W + 1);
+      b = run_pass<L, 32, C, true, PP>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps, P, S,
+                                       rb + (int64_t)si * p.rb_cols, rb + (int64_t)so * p.rb_cols, prog + si,
+                                       prog + so, b);
+    }
+#pragma unroll
+    for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
+    if (lane == 0) sred[warp] = b;
+    team_bar(team, W);
+    if (wt == 0 && lane == 0) {
+      uint32_t bb = sred[team * W];
+      for (int i = 1; i < W; ++i) bb = L::max2(bb, sred[team * W + i]);
+      const int limit = 32767 - p.max_w;
+      const int s0 = 2 * item, s1 = 2 * item + 1;
+      const int lo = (int)(int16_t)(bb & 0xffffu), hi = (int)(int16_t)(bb >> 16);
+      if (lo >= limit) p.ovf_list[atomicAdd(p.ovf_count, 1)] = s0; else p.scores[p.perm[s0]] = lo;
+      if (s1 < p.n_seqs) {
+        if (hi >= limit) p.ovf_list[atomicAdd(p.ovf_count, 1)] = s1; else p.scores[p.perm[s1]] = hi;
+      }
+    }
+  }
+}
+
+template <int C, int NT, bool PP>
+cudaError_t launch_search_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st) {
+  k_search_t<C, NT, PP><<<grid, NT, smem_bytes, st>>>(p);
+  return cudaGetLastError();
+}
+
+template <int C, int NT, bool PP>
+cudaError_t configure_tmode(int smem_bytes, int* blocks_per_sm) {
+  cudaError_t e =
+      cudaFuncSetAttribute(k_search_t<C, NT, PP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+  if (e != cudaSuccess) return e;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search_t<C, NT, PP>, NT, smem_bytes);
 }
 
 template <class L, int G, int Rs, int Rl, int NT, bool PP>

@@ -52,7 +52,8 @@ struct SearchParams {
   int32_t* scores;           // caller order, int32
   // work partition: items [0, n_long) run in team (intra-task) mode, [n_long, n_pairs) in
   // group (inter-task) mode.  For the 32-bit recompute kernel items come from item_list.
-  int n_long;
+  int n_long;                // team-mode items (pairs [0, n_long)); 0 when T-mode takes them
+  int short_begin;           // first pair of the group-mode (short) range
   const int32_t* item_list;  // s32 recompute: sorted sequence positions (nullptr otherwise)
   const int32_t* item_count; // s32 recompute: device count
   int32_t* work;             // [0] team-item counter, [1] group-item counter
@@ -88,6 +89,34 @@ cudaError_t configure_kernel(const KernelConfig& cfg, int smem_bytes, int* block
 int menu_size();
 KernelConfig menu_entry(int i);
 KernelConfig recompute_config();
+
+// T-mode (transposed long-sequence kernel, sw_engine.cuh k_search_t): C database positions
+// per lane, one CTA team of up to kTmodeThreads / 32 warps per long pair.
+constexpr int kTmodeC = 16;
+constexpr int kTmodeThreads = 256;
+struct TParams {
+  const int8_t* matrix;      // A x A, [query][db]
+  int A, rho, sigma, max_w, pad_letter;
+  const uint16_t* qpair;     // query as (q | q << 8), qcols + kPadCols entries, pad beyond m
+  int qcols;                 // query length rounded up to 8
+  const uint16_t* cols;
+  const int64_t* pair_off;
+  const int32_t* pair_ncols;
+  int n_items;               // long pairs [0, n_items)
+  int n_seqs;
+  const int32_t* perm;
+  int32_t* scores;
+  int32_t* ovf_list;
+  int32_t* ovf_count;
+  int32_t* work;
+  int warps;                 // warps used per CTA (<= NT / 32, bounded by shared memory)
+  int team_warps;            // warps per team (divides warps)
+  uint2* rb; int64_t rb_cols;   // per (CTA, team): team_warps + 1 slots
+};
+
+cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st);
+cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm);
+cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, int pad, cudaStream_t st);
 
 // Profile image build: byte(rep, a, i) = (i < m && a < A) ? W[q_i][a] + rho : -128.
 cudaError_t launch_profile(uint8_t* blob, const ProfLayout& L, const uint8_t* q, int m, const int8_t* W, int A,

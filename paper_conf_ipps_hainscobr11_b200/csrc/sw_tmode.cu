@@ -1,0 +1,29 @@
+// sw_tmode.cu — instantiation of the transposed long-sequence kernel (k_search_t) and the
+// query-stream builder it reads.
+#include "sw_engine.cuh"
+#include "sw_internal.h"
+
+namespace swb {
+
+// qpair[i] = q_i | q_i << 8 for i < m, the pad letter pair beyond (qcols + kPadCols entries)
+__global__ void k_qpair(uint16_t* __restrict__ out, const uint8_t* __restrict__ q, int m, int n, int pad) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const int a = i < m ? (int)q[i] : pad;
+    out[i] = (uint16_t)(a | (a << 8));
+  }
+}
+
+cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, int pad, cudaStream_t st) {
+  k_qpair<<<(n + 255) / 256, 256, 0, st>>>(out, q, m, n, pad);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st) {
+  return launch_search_tmode<kTmodeC, kTmodeThreads, true>(p, grid, smem_bytes, st);
+}
+
+cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm) {
+  return configure_tmode<kTmodeC, kTmodeThreads, true>(smem_bytes, blocks_per_sm);
+}
+
+}  // namespace swb

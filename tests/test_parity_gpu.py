@@ -77,6 +77,24 @@ def test_every_config_both_regimes(menu):
             _assert_equal(out, ref, db, f"menu={menu} m={m} T={T}")
 
 
+@pytest.mark.parametrize("mode", ["team", "t8", "t2", "t1"])
+@pytest.mark.parametrize("m", [1, 37, 144, 567, 1500])
+def test_long_sequence_modes(mode, m):
+    """Both long-sequence paths (team: strips of query rows; t: transposed, strips of the
+    database sequence) on ragged long sequences, incl. the 35,213 maximum and lengths just
+    around a strip multiple (512 positions per T-mode strip)."""
+    rng = np.random.default_rng(77 + m)
+    lens = np.concatenate([[35213, 512, 511, 513, 1024, 3072, 3073], rng.integers(3000, 12000, size=9),
+                           rng.integers(0, 100, size=5)])
+    db = _db_from_lengths(lens, seed=300 + m, extra=True)
+    q = gen.make_query(m, seed=900 + m)
+    ref = _oracle(q, BLOSUM62, 10, 2, db)
+    for T in (0, 3000):
+        env = {"SW_LONG_MODE": "team"} if mode == "team" else {"SW_LONG_MODE": "t", "SW_T_TEAM": mode[1:]}
+        out, st = _gpu(q, BLOSUM62, 10, 2, db, T, env=env)
+        _assert_equal(out, ref, db, f"mode={mode} m={m} T={T}")
+
+
 @pytest.mark.parametrize("team", [1, 2, 3, 5])
 def test_team_mode_multi_warp(team):
     """Intra-task path with several warps chained over strips (progress-flag hand-off)."""
@@ -85,7 +103,8 @@ def test_team_mode_multi_warp(team):
     db = _db_from_lengths(lens, seed=40 + team)
     q = gen.make_query(1500, seed=5 + team)
     ref = _oracle(q, BLOSUM62, 10, 2, db)
-    out, _ = _gpu(q, BLOSUM62, 10, 2, db, 0, env={"SW_FORCE_MENU": 8, "SW_FORCE_TEAM_WARPS": team})
+    out, _ = _gpu(q, BLOSUM62, 10, 2, db, 0, env={"SW_FORCE_MENU": 8, "SW_FORCE_TEAM_WARPS": team,
+                                                  "SW_LONG_MODE": "team"})
     _assert_equal(out, ref, db, f"team={team}")
 
 
