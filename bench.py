@@ -212,7 +212,7 @@ def bench_ours(args, rank, world, local_rank):
         dist.barrier()
     qs, db, lens_all, mat, rho, sigma, T = make_workload(args.config, rank, world)
     if args.threshold is not None:
-        T = args.threshold
+        T = -1 if str(args.threshold) == "auto" else int(args.threshold)
     W = MATRICES[mat]
     nq = len(qs)
     from paper_conf_ipps_hainscobr11_b200.dist import ScoreGather, shard_size_bound
@@ -366,7 +366,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--config", default="C2")
-    ap.add_argument("--threshold", type=int, default=None)
+    ap.add_argument("--threshold", default=None, help="length threshold T (default: the config's, 3072); 'auto' = SW_AUTO_THRESHOLD")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()

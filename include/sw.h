@@ -52,6 +52,10 @@ enum {
 #define SW_MAX_QUERY_LEN (1 << 16)  /* 1 <= query_len <= 65536 */
 #define SW_MAX_SEQ_LEN ((1 << 20) - 64)  /* every database sequence length <= 1,048,512 */
 
+/* length_threshold value asking the library to choose the inter/intra-task threshold itself
+ * (§VI "automatic detection of the optimal threshold value"). */
+#define SW_AUTO_THRESHOLD (-1)
+
 /* Create a handle for one query and one scoring scheme (§II: q, w, rho, sigma).
  *   query[query_len]      codes < alphabet_size, 1 <= query_len <= SW_MAX_QUERY_LEN
  *   matrix[A*A]           int8, row = query symbol, column = database symbol
@@ -81,6 +85,9 @@ int sw_load_db(sw_handle h, const uint8_t* residues, int64_t total_residues,
  *   database sequence length is below 3072, the inter-task kernel is used. Otherwise,
  *   the intra-task kernel is used.").  Scores do not depend on T. */
 int sw_search(sw_handle h, int32_t* scores_out, int32_t length_threshold);
+/* (length_threshold == SW_AUTO_THRESHOLD: chosen per query by the library's time model;
+ * sw_last_threshold reports the value used by the last query.) */
+int32_t sw_last_threshold(sw_handle h);
 
 /* Same, stream-ordered: d_scores_out is a DEVICE int32[num_seqs] (e.g. a torch tensor);
  * cuda_stream is a cudaStream_t (NULL = legacy default stream).  Returns after enqueueing. */

@@ -20,8 +20,10 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libsw_b200.so")
 
 SW_OK, SW_E_INVALID, SW_E_STATE, SW_E_NOMEM, SW_E_CUDA, SW_E_UNSUPPORTED = range(6)
+SW_AUTO_THRESHOLD = -1
 EXPORTED = ["sw_create", "sw_set_query", "sw_load_db", "sw_search", "sw_search_async",
-            "sw_search_batch", "sw_search_batch_async", "sw_last_stats", "sw_last_kernel_ms", "sw_destroy",
+            "sw_search_batch", "sw_search_batch_async", "sw_last_stats", "sw_last_kernel_ms", "sw_last_threshold",
+            "sw_destroy",
             "sw_strerror", "sw_last_error", "sw_version"]
 
 _lib = None
@@ -51,6 +53,8 @@ def load_library(path: str = LIB_PATH):
     L.sw_search_batch_async.argtypes = [vp, vp, vp, i32, vp, i32, vp]
     L.sw_last_stats.argtypes = [vp, vp]
     L.sw_last_kernel_ms.argtypes = [vp, vp]
+    L.sw_last_threshold.argtypes = [vp]
+    L.sw_last_threshold.restype = ctypes.c_int32
     L.sw_destroy.argtypes = [vp]
     L.sw_destroy.restype = None
     L.sw_strerror.argtypes = [ctypes.c_int]
@@ -184,6 +188,9 @@ class SmithWaterman:
 
     def kernel_ms(self) -> dict:
         return sw_last_kernel_ms(self.h)
+
+    def last_threshold(self) -> int:
+        return int(load_library().sw_last_threshold(self.h))
 
     def close(self):
         if self.h:

@@ -56,6 +56,7 @@ struct sw_handle_s {
   std::vector<int32_t> h_pair_ncols;
   std::vector<int64_t> pair_cols_prefix;  // prefix sums of h_pair_ncols
   KernelConfig last_cfg{};
+  int32_t last_threshold = 0;
   uint16_t* d_cols = nullptr;
   int64_t* d_pair_off = nullptr;
   int32_t* d_pair_ncols = nullptr;
@@ -137,6 +138,8 @@ struct Plan {
   ProfLayout rl;       // recompute blob (team image only)
   int r_prof_bytes;
   int grid, rgrid;
+  double cost;         // estimated cycles of the main launch
+  double thr, tail_s;  // its throughput term and the critical path of the longest short item
 };
 
 int team_warps_for(int passes, int warps) {
@@ -195,8 +198,9 @@ int make_plan(sw_handle h, int m, const Split& sp, Plan* pl) {
     const double tail_l = sp.n_long ? (sp.long_max_cols + 31.0) * ((lt.strips + W - 1) / W) * il / kWarpIssue : 0.0;
     const double tail_s = sp.n_short ? (sp.short_max_cols + c.G - 1.0) * lg.strips * is / kWarpIssue : 0.0;
     const double cost = std::max(thr, std::max(tail_l, tail_s));
-    if (cost < best) { best = cost; best_i = i; }
+    if (cost < best) { best = cost; best_i = i; pl->thr = thr; pl->tail_s = tail_s; }
   }
+  pl->cost = best;
   // test hooks: force a menu entry / team size (used by the parity tests to cover every
   // compiled configuration; never needed for correctness)
   if (const char* f = getenv("SW_FORCE_MENU")) {
@@ -253,12 +257,10 @@ int validate_query(sw_handle h, const uint8_t* q, int32_t m) {
   return SW_OK;
 }
 
-// Enqueue one query (device query pointer) on slot s; scores to d_out (device, caller order).
-int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t* d_out, int32_t T,
-                  int32_t* h_ovf, cudaEvent_t* ev) {
-  // regime split: sorted_len is descending; long = n >= T (§II-B)
+// regime split: sorted_len is descending; long = n >= T (§II-B)
+Split make_split(sw_handle h, int64_t T, int64_t* n_long_seqs_out) {
   const int64_t n_long_seqs =
-      std::lower_bound(h->sorted_len.begin(), h->sorted_len.end(), (int64_t)T, std::greater_equal<int64_t>()) -
+      std::lower_bound(h->sorted_len.begin(), h->sorted_len.end(), T, std::greater_equal<int64_t>()) -
       h->sorted_len.begin();
   const int n_long = (int)((n_long_seqs + 1) / 2);
   Split sp;
@@ -268,6 +270,43 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   sp.short_cols = h->pair_cols_prefix[h->n_pairs] - sp.long_cols;
   sp.long_max_cols = n_long ? h->h_pair_ncols[0] : 0;
   sp.short_max_cols = sp.n_short ? h->h_pair_ncols[n_long] : 0;
+  if (n_long_seqs_out) *n_long_seqs_out = n_long_seqs;
+  return sp;
+}
+
+// Automatic inter/intra-task threshold (§VI: "characterize
+// the relative performance of the inter-task and intra-task kernels based on the mean and
+// maximum lengths ... during the database preprocessing step, we can find the transition
+// point").  Measured on B200 (profiles/r01_sweep_*.jsonl): the group (inter-task) path is the
+// faster one per cell, and long sequences only hurt it through the critical path of the
+// longest items (the paper's Fig.2 load-balance effect).  So the threshold is the LARGEST
+// candidate for which the longest short item still finishes within the group launch's
+// throughput time; everything longer goes to the long-sequence path.
+int64_t choose_threshold(sw_handle h, int m) {
+  const int64_t maxlen = h->sorted_len.empty() ? 0 : h->sorted_len[0];
+  const int64_t cands[] = {maxlen + 1, 16384, 12288, 8192, 6144, 4096, 3072, 2048, 1536, 1024, 768, 512};
+  const std::string saved = h->err;
+  int64_t chosen = 512;
+  for (int64_t T : cands) {
+    if (T > maxlen + 1) continue;
+    Split sp = make_split(h, T, nullptr);
+    sp.n_long = 0; sp.long_cols = 0; sp.long_max_cols = 0;   // the group launch alone
+    Plan pl;
+    if (make_plan(h, m, sp, &pl)) continue;
+    if (pl.tail_s <= 0.8 * pl.thr) { chosen = T; break; }
+  }
+  h->err = saved;
+  return chosen;
+}
+
+// Enqueue one query (device query pointer) on slot s; scores to d_out (device, caller order).
+int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t* d_out, int32_t T,
+                  int32_t* h_ovf, cudaEvent_t* ev) {
+  if (T == SW_AUTO_THRESHOLD) T = (int32_t)std::min<int64_t>(choose_threshold(h, m), INT32_MAX);
+  h->last_threshold = T;
+  int64_t n_long_seqs = 0;
+  const Split sp = make_split(h, T, &n_long_seqs);
+  const int n_long = sp.n_long;
   Plan pl;
   int rc = make_plan(h, m, sp, &pl);
   if (rc) return rc;
@@ -615,7 +654,8 @@ int sw_search_batch_async(sw_handle h, const uint8_t* queries, const int64_t* q_
   if (!h) return SW_E_INVALID;
   if (!h->db_loaded) return fail(h, SW_E_STATE, "sw_load_db has not been called");
   if (num_queries < 0 || !q_offsets || (num_queries > 0 && !queries)) return fail(h, SW_E_INVALID, "bad query batch");
-  if (length_threshold < 0) return fail(h, SW_E_INVALID, "length_threshold < 0");
+  if (length_threshold < 0 && length_threshold != SW_AUTO_THRESHOLD)
+    return fail(h, SW_E_INVALID, "length_threshold < 0 (use SW_AUTO_THRESHOLD for automatic)");
   if (h->n_seqs > 0 && num_queries > 0 && !d_scores_out) return fail(h, SW_E_INVALID, "d_scores_out is NULL");
   if (q_offsets[0] != 0) return fail(h, SW_E_INVALID, "q_offsets[0] != 0");
   for (int k = 0; k < num_queries; ++k) {
@@ -676,6 +716,8 @@ int sw_last_stats(sw_handle h, int64_t out[4]) {
   out[3] = h->stat_launches;
   return SW_OK;
 }
+
+int32_t sw_last_threshold(sw_handle h) { return h ? h->last_threshold : -1; }
 
 int sw_last_kernel_ms(sw_handle h, double out[2]) {
   if (!h || !out) return SW_E_INVALID;

@@ -1,0 +1,119 @@
+"""C-ABI contract on the GPU (include/sw.h): one test per error code / state rule, ownership
+(inputs copied), the device-pointer stream-ordered entry points and the statistics calls."""
+import ctypes
+
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_ipps_hainscobr11_b200 as swp
+from workloads import gen
+from workloads.matrices import BLOSUM62
+
+pytestmark = pytest.mark.gpu
+
+
+def _db(n=200, seed=4):
+    return gen.build_database(gen.sp_lengths(n, seed=seed), seed)
+
+
+def test_search_before_load_is_state_error():
+    h = swp.sw_create(gen.make_query(50), BLOSUM62, 10, 2)
+    try:
+        with pytest.raises(swp.SWError) as e:
+            swp.sw_search(h, 1, 3072)
+        assert e.value.status == swp.SW_E_STATE
+    finally:
+        swp.sw_destroy(h)
+
+
+def test_invalid_arguments():
+    L = swp.load_library()
+    h = swp.sw_create(gen.make_query(50), BLOSUM62, 10, 2)
+    try:
+        res = np.zeros(10, np.uint8)
+        bad_off = np.array([0, 5, 3, 10], np.int64)          # not non-decreasing
+        assert L.sw_load_db(h, res.ctypes.data, 10, bad_off.ctypes.data, 3) == swp.SW_E_INVALID
+        bad_off2 = np.array([1, 5, 10], np.int64)            # offsets[0] != 0
+        assert L.sw_load_db(h, res.ctypes.data, 10, bad_off2.ctypes.data, 2) == swp.SW_E_INVALID
+        bad_res = np.full(10, 30, np.uint8)                   # code >= alphabet
+        off = np.array([0, 10], np.int64)
+        assert L.sw_load_db(h, bad_res.ctypes.data, 10, off.ctypes.data, 1) == swp.SW_E_INVALID
+        assert b"alphabet" in L.sw_last_error(h)
+        swp.sw_load_db(h, np.zeros(10, np.uint8), off)
+        out = np.zeros(1, np.int32)
+        assert L.sw_search(h, out.ctypes.data, -2) == swp.SW_E_INVALID   # T < 0 (and not SW_AUTO_THRESHOLD)
+        assert L.sw_search(h, None, 10) == swp.SW_E_INVALID             # NULL output
+        q = np.array([1, 2, 99], np.uint8)
+        assert L.sw_set_query(h, q.ctypes.data, 3) == swp.SW_E_INVALID   # bad query code
+        assert L.sw_set_query(h, q.ctypes.data, 0) == swp.SW_E_INVALID   # empty query
+    finally:
+        swp.sw_destroy(h)
+
+
+def test_inputs_are_copied_and_reload_replaces_db():
+    db = _db()
+    q = gen.make_query(120)
+    h = swp.sw_create(q, BLOSUM62, 10, 2)
+    try:
+        res = db.residues.copy()
+        swp.sw_load_db(h, res, db.offsets)
+        res[:] = 0                      # caller reuses its buffer: the library owns a copy
+        q[:] = 0
+        out = swp.sw_search(h, db.num_seqs, 3072)
+        ref = oracle.scores(gen.make_query(120), BLOSUM62, 10, 2, db.residues, db.offsets)
+        assert np.array_equal(out, ref)
+        db2 = _db(50, seed=9)
+        swp.sw_load_db(h, db2.residues, db2.offsets)
+        out2 = swp.sw_search(h, db2.num_seqs, 3072)
+        assert out2.shape == (50,)
+        assert np.array_equal(out2, oracle.scores(gen.make_query(120), BLOSUM62, 10, 2, db2.residues, db2.offsets))
+    finally:
+        swp.sw_destroy(h)
+
+
+def test_async_device_pointer_and_stream():
+    import torch
+    db = _db()
+    q = gen.make_query(333)
+    with swp.SmithWaterman(q, BLOSUM62, 10, 2) as sw:
+        sw.load_db(db.residues, db.offsets)
+        st = torch.cuda.Stream()
+        out = torch.full((db.num_seqs,), -7, dtype=torch.int32, device="cuda")
+        swp.sw_search_async(sw.h, out.data_ptr(), 3072, st.cuda_stream)
+        st.synchronize()
+        ref = oracle.scores(q, BLOSUM62, 10, 2, db.residues, db.offsets)
+        assert np.array_equal(out.cpu().numpy(), ref)
+        # batch into a device tensor, joined back into the caller's stream
+        qs = [gen.make_query(L) for L in (144, 375, 5)]
+        outb = torch.full((3, db.num_seqs), -1, dtype=torch.int32, device="cuda")
+        sw.search_batch_into(qs, outb.data_ptr(), 3072, st.cuda_stream)
+        st.synchronize()
+        for k, qq in enumerate(qs):
+            assert np.array_equal(outb[k].cpu().numpy(), oracle.scores(qq, BLOSUM62, 10, 2, db.residues, db.offsets))
+        stats = sw.stats()
+        assert stats["launches"] > 0 and stats["recomputed_s32"] == 0
+        km = sw.kernel_ms()
+        assert km["search_ms"] > 0
+
+
+def test_unsupported_parameter_ranges():
+    with pytest.raises(swp.SWError) as e:
+        swp.sw_create(gen.make_query(10), BLOSUM62, 120, 1)     # 120 + 11 > 127: int8 profile range
+    assert e.value.status == swp.SW_E_UNSUPPORTED
+    # a query whose profile cannot be staged in shared memory is refused, never computed on the CPU
+    h = swp.sw_create(gen.make_query(20000), BLOSUM62, 10, 2)
+    try:
+        db = _db(20)
+        swp.sw_load_db(h, db.residues, db.offsets)
+        with pytest.raises(swp.SWError) as e:
+            swp.sw_search(h, db.num_seqs, 3072)
+        assert e.value.status == swp.SW_E_UNSUPPORTED
+    finally:
+        swp.sw_destroy(h)
+
+
+def test_version_and_null_destroy():
+    L = swp.load_library()
+    assert L.sw_version().startswith(b"sw_b200")
+    L.sw_destroy(ctypes.c_void_p())

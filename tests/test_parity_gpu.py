@@ -283,3 +283,22 @@ def test_c2_full_size_sampled():
         got = outb[k][sample]
         assert np.array_equal(got, ref), (k, np.nonzero(got != ref)[0][:10])
         assert (outb[k] >= 0).all()
+
+
+# ------------------------------------------------------------------ automatic threshold (f1)
+@pytest.mark.parametrize("cfg", ["C1", "C3"])
+def test_auto_threshold_parity(cfg):
+    if cfg == "C1":
+        wl = gen.config("C1", n_override=3000)
+        db, q = wl.db, wl.queries[0]
+    else:
+        lens = gen.long_lengths(64, seed=3, max_len=9000)
+        q = gen.make_query(567)
+        db = gen.build_database(lens, 3, [q])
+    ref = _oracle(q, BLOSUM62, 10, 2, db)
+    with swp.SmithWaterman(q, BLOSUM62, 10, 2) as sw:
+        sw.load_db(db.residues, db.offsets)
+        out = sw.search(swp.SW_AUTO_THRESHOLD)
+        T = sw.last_threshold()
+    _assert_equal(out, ref, db, f"auto T={T}")
+    assert T >= 0

@@ -15,7 +15,7 @@ from workloads import gen  # noqa: E402
 from workloads.matrices import BLOSUM62  # noqa: E402
 
 cfg, m = sys.argv[1], int(sys.argv[2])
-Ts = [int(x) for x in sys.argv[3].split(",")]
+Ts = [int(x) if x != "auto" else -1 for x in sys.argv[3].split(",")]
 if cfg == "C3":
     lens = gen.long_lengths(4096, seed=3)
     db = gen.build_database(lens, 3, None)
@@ -33,6 +33,9 @@ def subset(mask):
     return res, off, int(L[idx].sum())
 
 
+LAST_T = [None]
+
+
 def timed(res, off, T):
     if off.shape[0] <= 1 or off[-1] == 0:
         return 0.0
@@ -40,17 +43,21 @@ def timed(res, off, T):
         sw.load_db(res, off)
         sw.search(T)
         sw.search(T)
+        LAST_T[0] = sw.last_threshold()
         return sw.kernel_ms()["search_ms"]
 
 
 full_ms = {}
 for T in Ts:
     t_all = timed(db.residues, db.offsets, T)
+    auto = T < 0
+    if auto:
+        T = LAST_T[0]
     res_l, off_l, n_l = subset(L >= T)
     res_s, off_s, n_s = subset(L < T)
     t_l = timed(res_l, off_l, T)
     t_s = timed(res_s, off_s, T)
-    line = {"config": cfg, "m": m, "T": T, "frac_seqs_long": round(float((L >= T).mean()), 5),
+    line = {"config": cfg, "m": m, "T": T, "auto": auto, "frac_seqs_long": round(float((L >= T).mean()), 5),
             "frac_res_long": round(n_l / max(1, int(L.sum())), 5), "ms_total": round(t_all, 3),
             "gcups_total": round(m * int(L.sum()) / t_all / 1e6, 1) if t_all else None,
             "gcups_long_only": round(m * n_l / t_l / 1e6, 1) if t_l else None,
