@@ -190,7 +190,11 @@ int make_plan(sw_handle h, int m, const Split& sp, Plan* pl) {
     // several strips in group mode are only efficient for whole-warp chains: with G < 32 the
     // strip-boundary row traffic per cell grows by 32 / G and its latency dominates (measured)
     if (lg.strips > 1 && c.G < 32) continue;
-    const double is = 6.5 * c.Rs + 24.0, il = 6.5 * c.Rl + 40.0;   // ALU instructions per step
+    // ALU instructions per step; a config with more resident warps per scheduler hides the
+    // 2 x 4.4-cycle F/H dependency chain better (measured: 3 warps ~2.5 % faster than 2)
+    const double wps = c.threads / 128.0;
+    const double lat = 1.0 - 0.025 * std::min(2.0, std::max(0.0, wps - 2.0));
+    const double is = (6.5 * c.Rs + 24.0) * lat, il = (6.5 * c.Rl + 40.0) * lat;
     const int W = team_warps_for(lt.strips, c.threads / 32);
     const double gsteps = ((double)sp.short_cols + (double)sp.n_short * (c.G - 1)) * lg.strips / (32 / c.G);
     const double tsteps = ((double)sp.long_cols + 31.0 * sp.n_long) * lt.strips;
@@ -310,6 +314,21 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   Plan pl;
   int rc = make_plan(h, m, sp, &pl);
   if (rc) return rc;
+  // Long pairs: T-mode (strips along the database sequence) when the query is short enough
+  // that team mode would have few query strips to spread over warps; team mode otherwise.
+  // SW_LONG_MODE=team|t overrides (tests).
+  bool use_t = n_long > 0 && pl.long_passes <= 2;
+  if (const char* f = getenv("SW_LONG_MODE")) {
+    if (!strcmp(f, "team")) use_t = false;
+    if (!strcmp(f, "t")) use_t = n_long > 0;
+  }
+  if (use_t) {
+    // the main launch then only sees the short pairs: plan it for them
+    Split ss = sp;
+    ss.n_long = 0; ss.long_cols = 0; ss.long_max_cols = 0;
+    rc = make_plan(h, m, ss, &pl);
+    if (rc) return rc;
+  }
   h->last_cfg = pl.cfg;
 
   // scratch: profile, overflow list, row buffers
@@ -328,7 +347,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   if (pl.short_passes > 1 && max_cols_short > 0)
     rbg = (size_t)pl.grid * (pl.cfg.threads / 32) * (32 / G) * max_cols_short * sizeof(uint2);
   size_t rbt = 0;
-  if (pl.long_passes > 1 && n_long > 0) {
+  if (pl.long_passes > 1 && n_long > 0 && !use_t) {
     const int nteams = (pl.cfg.threads / 32) / pl.team_warps;
     rbt = (size_t)pl.grid * nteams * (pl.team_warps + 1) * max_cols_all * sizeof(uint2);
   }
@@ -341,14 +360,6 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   rc = grow(h, &s.d_rb_team, &s.rb_team_cap, rbt, "alloc team row buffers", s.stream);
   if (rc) return rc;
 
-  // Long pairs: T-mode (strips along the database sequence) when the query is short enough
-  // that team mode would have few query strips to spread over warps; team mode otherwise.
-  // SW_LONG_MODE=team|t overrides (tests).
-  bool use_t = n_long > 0 && pl.long_passes <= 2;
-  if (const char* f = getenv("SW_LONG_MODE")) {
-    if (!strcmp(f, "team")) use_t = false;
-    if (!strcmp(f, "t")) use_t = n_long > 0;
-  }
   const int qcols = (int)round_up(m, 8);
   const int wp_bytes = (int)round_up((int64_t)(h->A + 1) * 32, 128);
   const int per_warp = 2 * (h->A + 1) * 32 * kTmodeC;
