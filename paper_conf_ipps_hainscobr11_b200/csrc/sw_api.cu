@@ -291,12 +291,24 @@ int64_t choose_threshold(sw_handle h, int m) {
   const int64_t cands[] = {maxlen + 1, 16384, 12288, 8192, 6144, 4096, 3072, 2048, 1536, 1024, 768, 512};
   const std::string saved = h->err;
   int64_t chosen = 512;
+  // whole-warp chains at the paper's default threshold?  (see below)
+  bool g32 = false;
+  {
+    Split sp = make_split(h, 3072, nullptr);
+    sp.n_long = 0; sp.long_cols = 0; sp.long_max_cols = 0;
+    Plan pl;
+    if (!make_plan(h, m, sp, &pl)) g32 = pl.cfg.G == 32;
+  }
   for (int64_t T : cands) {
     if (T > maxlen + 1) continue;
     Split sp = make_split(h, T, nullptr);
     sp.n_long = 0; sp.long_cols = 0; sp.long_max_cols = 0;   // the group launch alone
     Plan pl;
     if (make_plan(h, m, sp, &pl)) continue;
+    // thresholds above the paper's default are taken only with whole-warp chains (G = 32):
+    // with sub-warp chains the long short-items run on a fraction of a warp and the measured
+    // tail is worse than the model's (profiles/r01_query_sweep_auto.jsonl)
+    if (T > 3072 && (!g32 || pl.cfg.G < 32)) continue;
     if (pl.tail_s <= 0.8 * pl.thr) { chosen = T; break; }
   }
   h->err = saved;

@@ -55,7 +55,7 @@ def _assert_equal(gpu, ref, db, what=""):
 
 
 # ------------------------------------------------------------------ every configuration, both regimes
-MENU = [i for i in range(21) if i != 11]  # s16x2 entries of csrc/gen_menu.py (11 is the s32 recompute)
+MENU = [i for i in range(28) if i != 11]  # s16x2 entries of csrc/gen_menu.py (11 is the s32 recompute)
 
 
 @pytest.mark.parametrize("menu", MENU)
