@@ -36,7 +36,9 @@ struct QuerySlot {
   uint16_t* d_qpair = nullptr;    // T-mode query stream
   size_t qpair_cap = 0;
   cudaStream_t stream = nullptr;
+  cudaStream_t aux = nullptr;      // T-mode launch, concurrent with the group launch
   cudaEvent_t done = nullptr;
+  cudaEvent_t fork = nullptr, join = nullptr;
 };
 
 }  // namespace
@@ -245,6 +247,9 @@ int ensure_slots(sw_handle h, int n) {
   while ((int)h->slots.size() < n) {
     QuerySlot s;
     SW_CUDA(h, cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking));
+    SW_CUDA(h, cudaStreamCreateWithFlags(&s.aux, cudaStreamNonBlocking));
+    SW_CUDA(h, cudaEventCreateWithFlags(&s.fork, cudaEventDisableTiming));
+    SW_CUDA(h, cudaEventCreateWithFlags(&s.join, cudaEventDisableTiming));
     SW_CUDA(h, cudaEventCreateWithFlags(&s.done, cudaEventDisableTiming));
     SW_CUDA(h, cudaMalloc(&s.d_work, 4 * sizeof(int32_t)));
     SW_CUDA(h, cudaMalloc(&s.d_ovf_count, sizeof(int32_t)));
@@ -281,35 +286,41 @@ Split make_split(sw_handle h, int64_t T, int64_t* n_long_seqs_out) {
 // Automatic inter/intra-task threshold (§VI: "characterize
 // the relative performance of the inter-task and intra-task kernels based on the mean and
 // maximum lengths ... during the database preprocessing step, we can find the transition
-// point").  Measured on B200 (profiles/r01_sweep_*.jsonl): the group (inter-task) path is the
-// faster one per cell, and long sequences only hurt it through the critical path of the
-// longest items (the paper's Fig.2 load-balance effect).  So the threshold is the LARGEST
-// candidate for which the longest short item still finishes within the group launch's
-// throughput time; everything longer goes to the long-sequence path.
+// point").  For each candidate T the planner's time model gives the group (inter-task)
+// launch's throughput time and the critical path of its longest item; the long (intra-task)
+// pairs run concurrently in T-mode at ~2.2x the group cost per cell (measured,
+// profiles/r01_sweep_*.jsonl).  Estimated time = max(throughput of both launches,
+// group tail / 0.8); the cheapest candidate wins (ties: the larger T).
 int64_t choose_threshold(sw_handle h, int m) {
   const int64_t maxlen = h->sorted_len.empty() ? 0 : h->sorted_len[0];
   const int64_t cands[] = {maxlen + 1, 16384, 12288, 8192, 6144, 4096, 3072, 2048, 1536, 1024, 768, 512};
   const std::string saved = h->err;
-  int64_t chosen = 512;
-  // whole-warp chains at the paper's default threshold?  (see below)
-  bool g32 = false;
+  int64_t chosen = 3072;
+  double best = 1e300;
+  // group cost per database column, from the plan with every pair in the group launch
+  double per_col = 0.0;
   {
-    Split sp = make_split(h, 3072, nullptr);
-    sp.n_long = 0; sp.long_cols = 0; sp.long_max_cols = 0;
+    Split sp = make_split(h, maxlen + 1, nullptr);
     Plan pl;
-    if (!make_plan(h, m, sp, &pl)) g32 = pl.cfg.G == 32;
+    if (!make_plan(h, m, sp, &pl) && sp.short_cols > 0) per_col = pl.thr * (2.7 / 2.0) / (double)sp.short_cols;
   }
   for (int64_t T : cands) {
     if (T > maxlen + 1) continue;
     Split sp = make_split(h, T, nullptr);
+    const double long_cols = (double)sp.long_cols;
     sp.n_long = 0; sp.long_cols = 0; sp.long_max_cols = 0;   // the group launch alone
     Plan pl;
-    if (make_plan(h, m, sp, &pl)) continue;
-    // thresholds above the paper's default are taken only with whole-warp chains (G = 32):
-    // with sub-warp chains the long short-items run on a fraction of a warp and the measured
-    // tail is worse than the model's (profiles/r01_query_sweep_auto.jsonl)
-    if (T > 3072 && (!g32 || pl.cfg.G < 32)) continue;
-    if (pl.tail_s <= 0.8 * pl.thr) { chosen = T; break; }
+    if (sp.n_short > 0 && make_plan(h, m, sp, &pl)) continue;
+    if (sp.n_short == 0) { pl.thr = 0.0; pl.tail_s = 0.0; }
+    // measured rates: the whole GPU sustains ~0.5 ALU warp-instructions / clock / scheduler
+    // (not the model's 2.7 / SM), and a tail warp ~0.15 (profiles/r01_ncu_*, query sweeps)
+    const double thr = pl.thr * (2.7 / 2.0), tail = pl.tail_s * (0.2 / 0.15);
+    const double thr_long = per_col * long_cols * 2.2;
+    const double cost = std::max(thr + thr_long, tail / 0.8);
+    if (getenv("SW_DEBUG_AUTO"))
+      fprintf(stderr, "auto m=%d T=%lld G=%d Rs=%d thr=%.3f long=%.3f tail=%.3f cost=%.3f ms\n", m, (long long)T,
+              pl.cfg.G, pl.cfg.Rs, thr / 1.965e6, thr_long / 1.965e6, tail / 1.965e6, cost / 1.965e6);
+    if (cost < best * 0.995) { best = cost; chosen = T; }
   }
   h->err = saved;
   return chosen;
@@ -431,7 +442,12 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   p.rb_team_cols = max_cols_all;
   SW_CUDA(h, cudaEventRecord(ev[0], st));
   if (use_t) {
+    // T-mode runs on the slot's second stream, concurrently with the group launch: its CTAs
+    // take every SM first (launched first), and as they run out of long pairs the group
+    // launch's CTAs take their SMs, so the longest long pair overlaps the short-pair work.
     SW_CUDA(h, launch_qpair(s.d_qpair, d_q, m, qcols + kPadCols, h->A, st));
+    SW_CUDA(h, cudaEventRecord(s.fork, st));
+    SW_CUDA(h, cudaStreamWaitEvent(s.aux, s.fork, 0));
     TParams t{};
     t.matrix = h->d_matrix;
     t.A = h->A;
@@ -462,9 +478,11 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
     t.team_warps = W;
     t.rb = s.d_rb_t;
     t.rb_cols = qcols + kPadCols;
-    SW_CUDA(h, launch_tmode(t, t_grid, t_smem, st));
+    SW_CUDA(h, launch_tmode(t, t_grid, t_smem, s.aux));
+    SW_CUDA(h, cudaEventRecord(s.join, s.aux));
   }
   SW_CUDA(h, launch_search(pl.cfg, p, pl.grid, pl.prof_bytes, st));
+  if (use_t) SW_CUDA(h, cudaStreamWaitEvent(st, s.join, 0));
   SW_CUDA(h, cudaEventRecord(ev[1], st));
 
   // exact 32-bit recompute of sequences whose 16-bit best reached 32767 - max_w
@@ -764,6 +782,9 @@ void sw_destroy(sw_handle h) {
     cudaFree(s.d_prof); cudaFree(s.d_work); cudaFree(s.d_ovf_count); cudaFree(s.d_ovf_list);
     cudaFree(s.d_rb_group); cudaFree(s.d_rb_team); cudaFree(s.d_query); cudaFree(s.d_rb_t); cudaFree(s.d_qpair);
     if (s.stream) cudaStreamDestroy(s.stream);
+    if (s.aux) { cudaStreamSynchronize(s.aux); cudaStreamDestroy(s.aux); }
+    if (s.fork) cudaEventDestroy(s.fork);
+    if (s.join) cudaEventDestroy(s.join);
     if (s.done) cudaEventDestroy(s.done);
   }
   cudaFree(h->d_matrix); cudaFree(h->d_cols); cudaFree(h->d_pair_off); cudaFree(h->d_pair_ncols);
