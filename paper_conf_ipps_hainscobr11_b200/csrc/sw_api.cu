@@ -200,7 +200,10 @@ int make_plan(sw_handle h, int m, const Split& sp, Plan* pl) {
     const int W = team_warps_for(lt.strips, c.threads / 32);
     const double gsteps = ((double)sp.short_cols + (double)sp.n_short * (c.G - 1)) * lg.strips / (32 / c.G);
     const double tsteps = ((double)sp.long_cols + 31.0 * sp.n_long) * lt.strips;
-    const double thr = (gsteps * is + tsteps * il) / kGpuIssue;
+    double thr = (gsteps * is + tsteps * il) / kGpuIssue;
+    // few items: the issue rate needs ~2 busy warps per scheduler (4 per SM)
+    const double active_warps = (double)sp.n_short / (32 / c.G) + (double)sp.n_long * W;
+    thr /= std::min(1.0, std::max(0.05, active_warps / (8.0 * h->num_sms)));
     const double tail_l = sp.n_long ? (sp.long_max_cols + 31.0) * ((lt.strips + W - 1) / W) * il / kWarpIssue : 0.0;
     const double tail_s = sp.n_short ? (sp.short_max_cols + c.G - 1.0) * lg.strips * is / kWarpIssue : 0.0;
     const double cost = std::max(thr, std::max(tail_l, tail_s));
@@ -288,7 +291,7 @@ Split make_split(sw_handle h, int64_t T, int64_t* n_long_seqs_out) {
 // maximum lengths ... during the database preprocessing step, we can find the transition
 // point").  For each candidate T the planner's time model gives the group (inter-task)
 // launch's throughput time and the critical path of its longest item; the long (intra-task)
-// pairs run concurrently in T-mode at ~2.2x the group cost per cell (measured,
+// pairs run concurrently in T-mode at ~1.8x the group cost per cell (measured,
 // profiles/r01_sweep_*.jsonl).  Estimated time = max(throughput of both launches,
 // group tail / 0.8); the cheapest candidate wins (ties: the larger T).
 int64_t choose_threshold(sw_handle h, int m) {
@@ -315,7 +318,7 @@ int64_t choose_threshold(sw_handle h, int m) {
     // measured rates: the whole GPU sustains ~0.5 ALU warp-instructions / clock / scheduler
     // (not the model's 2.7 / SM), and a tail warp ~0.15 (profiles/r01_ncu_*, query sweeps)
     const double thr = pl.thr * (2.7 / 2.0), tail = pl.tail_s * (0.2 / 0.15);
-    const double thr_long = per_col * long_cols * 2.2;
+    const double thr_long = per_col * long_cols * 1.8;
     const double cost = std::max(thr + thr_long, tail / 0.8);
     if (getenv("SW_DEBUG_AUTO"))
       fprintf(stderr, "auto m=%d T=%lld G=%d Rs=%d thr=%.3f long=%.3f tail=%.3f cost=%.3f ms\n", m, (long long)T,
@@ -468,14 +471,17 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
     t.ovf_count = s.d_ovf_count;
     t.work = s.d_work + 3;
     t.warps = t_warps;
-    // team size ~ strips of a typical long item (512 database positions per strip), so short
-    // long-items do not leave warps of a team idle: W in {1, 2, 4, 8}, W | t_warps
+    // Phase 1: pairs with >= big_strips strips (8192 positions) take the whole CTA as one
+    // team; phase 2: teams of W warps, W ~ a quarter of a typical pair's strips (fill and
+    // end-of-item waits grow as W^2 / strips), W in {1, 2, 4, 8}, W | t_warps.
     const double avg_strips = (double)sp.long_cols / std::max(1, n_long) / (32.0 * kTmodeC);
     int W = 1;
-    while (W * 2 <= t_warps && W * 2 <= avg_strips + 0.5 && t_warps % (W * 2) == 0) W *= 2;
+    while (W * 2 <= t_warps && W * 2 <= avg_strips / 4.0 + 0.5 && t_warps % (W * 2) == 0) W *= 2;
     if (const char* f = getenv("SW_T_TEAM")) W = std::max(1, std::min(t_warps, atoi(f)));
     while (t_warps % W) --W;
     t.team_warps = W;
+    t.big_strips = 16;
+    if (const char* f = getenv("SW_T_BIG")) t.big_strips = std::max(1, atoi(f));
     t.rb = s.d_rb_t;
     t.rb_cols = qcols + kPadCols;
     SW_CUDA(h, launch_tmode(t, t_grid, t_smem, s.aux));

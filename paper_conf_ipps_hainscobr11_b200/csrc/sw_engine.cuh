@@ -477,53 +477,40 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
 // pair's second sequence, chunk-major and conflict-free like the query profile) and the
 // residue stream is the query.  Strip boundaries (the last database position of a strip over
 // all query positions) go through the team row buffers with progress flags, as in team mode.
-template <int C, int NT, bool PP>
-__global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
+// One T-mode team (W warps) processing long pairs until the queue is exhausted.  first_item:
+// an item already taken for this team (or -1).  max_strips: a team of W warps only keeps items
+// with at most this many strips (> max_strips: the item is parked in *parked and the loop
+// returns, so that the CTA can regroup into smaller teams for the remaining, shorter items).
+template <int C, bool PP>
+__device__ __forceinline__ void t_team_loop(const TParams& p, const ChainConst& c, uint8_t* tab,
+                                            const int8_t* wp, int W, int team, int wt, int first_item,
+                                            int min_strips, int* parked, uint32_t* prog, uint2* rb,
+                                            int32_t* sitem, uint32_t* sred) {
   using L = LaneS16x2;
-  constexpr int kWarps = NT / 32;
   constexpr int CB = chunk_bytes<C>();
-  constexpr int LS = 32 * C;                  // letter stride of one strip table (bytes)
-  extern __shared__ __align__(128) uint8_t smem[];
-  __shared__ uint32_t sprog[2 * kWarps];
-  __shared__ uint32_t sred[kWarps];
-  __shared__ int32_t sitem[kWarps];
+  constexpr int LS = 32 * C;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int A1 = p.A + 1;
-  const int table_bytes = 2 * A1 * LS;        // lo + hi tables of one warp
-  int8_t* wp = reinterpret_cast<int8_t*>(smem);  // (A+1) x 32: w + rho, pad -> -128
-  uint8_t* tables = smem + ((A1 * 32 + 127) & ~127);
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  for (int t = threadIdx.x; t < A1 * 32; t += blockDim.x) {
-    const int a = t >> 5, d = t & 31;
-    int v = kPadValue;
-    if (a < p.A && d < p.A) v = (int)p.matrix[a * p.A + d] + p.rho;
-    wp[t] = (int8_t)v;
-  }
-  __syncthreads();
-  // teams of W warps (W | warps); several teams per CTA when long items have few strips
-  const int W = p.team_warps;
-  const int nteams = p.warps / W;
-  const int team = warp / W, wt = warp % W;
-  if (team >= nteams) return;
-  ChainConst c;
-  c.rho = p.rho;
-  c.sigma = p.sigma;
-  c.padpair = (uint32_t)p.pad_letter | ((uint32_t)p.pad_letter << 8);
-  uint8_t* tab = tables + warp * table_bytes;
   const int qsteps = (p.qcols + 31 + 3) & ~3;
-  uint32_t* prog = sprog + team * (W + 1);
-  uint2* rb = p.rb + ((int64_t)blockIdx.x * nteams + team) * (W + 1) * p.rb_cols;
+  int pending = first_item;
   for (;;) {
     team_bar(team, W);
     if (wt == 0 && lane == 0) {
-      sitem[team] = atomicAdd(p.work, 1);
+      const int it = pending >= 0 ? pending : atomicAdd(p.work, 1);
+      sitem[team] = it;
       for (int i = 0; i <= W; ++i) prog[i] = 0u;
     }
+    pending = -1;
     team_bar(team, W);
     const int item = sitem[team];
-    if (item >= p.n_items) break;
+    if (item >= p.n_items) return;
     const int ncols = p.pair_ncols[item];
-    const uint16_t* cp = p.cols + p.pair_off[item];
     const int S = (ncols + LS - 1) / LS;       // strips of the database pair
+    if (S < min_strips) {                      // too short for this team size: hand it back
+      if (wt == 0 && lane == 0) *parked = item;
+      return;
+    }
+    const uint16_t* cp = p.cols + p.pair_off[item];
     uint32_t b = 0;
     for (int P = wt; P < S; P += W) {
       // build this warp's strip tables: position pos = P*LS + lane*C + r
@@ -573,6 +560,52 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
       }
     }
   }
+}
+
+template <int C, int NT, bool PP>
+__global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
+  constexpr int kWarps = NT / 32;
+  constexpr int LS = 32 * C;
+  extern __shared__ __align__(128) uint8_t smem[];
+  __shared__ uint32_t sprog[2 * kWarps];
+  __shared__ uint32_t sred[kWarps];
+  __shared__ int32_t sitem[kWarps];
+  __shared__ int32_t sparked;
+  const int A1 = p.A + 1;
+  const int table_bytes = 2 * A1 * LS;        // lo + hi tables of one warp
+  int8_t* wp = reinterpret_cast<int8_t*>(smem);  // (A+1) x 32: w + rho, pad -> -128
+  uint8_t* tables = smem + ((A1 * 32 + 127) & ~127);
+  const int warp = threadIdx.x >> 5;
+  for (int t = threadIdx.x; t < A1 * 32; t += blockDim.x) {
+    const int a = t >> 5, d = t & 31;
+    int v = kPadValue;
+    if (a < p.A && d < p.A) v = (int)p.matrix[a * p.A + d] + p.rho;
+    wp[t] = (int8_t)v;
+  }
+  if (threadIdx.x == 0) sparked = -1;
+  __syncthreads();
+  if (warp >= p.warps) return;
+  ChainConst c;
+  c.rho = p.rho;
+  c.sigma = p.sigma;
+  c.padpair = (uint32_t)p.pad_letter | ((uint32_t)p.pad_letter << 8);
+  uint8_t* tab = tables + warp * table_bytes;
+  uint2* rb_cta = p.rb + (int64_t)blockIdx.x * (2 * p.warps) * p.rb_cols;
+  // Phase 1: one team of all warps for the longest pairs (items come longest-first), so the
+  // very long ones get the most parallelism; stops at the first pair with few strips.
+  // Phase 2: teams of team_warps for the rest — small teams waste less time in the pipeline
+  // fill and in the end-of-item barrier (T-mode ncu: 17 % barrier stalls with 8-warp teams).
+  if (p.warps > p.team_warps) {
+    t_team_loop<C, PP>(p, c, tab, wp, p.warps, 0, warp, -1, p.big_strips, &sparked, sprog, rb_cta, sitem, sred);
+    __syncthreads();
+  }
+  const int W = p.team_warps;
+  const int nteams = p.warps / W;
+  const int team = warp / W, wt = warp % W;
+  if (team >= nteams) return;
+  const int first = (team == 0) ? sparked : -1;
+  t_team_loop<C, PP>(p, c, tab, wp, W, team, wt, first, 0, nullptr, sprog + team * (W + 1),
+                     rb_cta + (int64_t)team * (W + 1) * p.rb_cols, sitem, sred);
 }
 
 template <int C, int NT, bool PP>

@@ -110,8 +110,9 @@ struct TParams {
   int32_t* ovf_count;
   int32_t* work;
   int warps;                 // warps used per CTA (<= NT / 32, bounded by shared memory)
-  int team_warps;            // warps per team (divides warps)
-  uint2* rb; int64_t rb_cols;   // per (CTA, team): team_warps + 1 slots
+  int team_warps;            // warps per team in phase 2 (divides warps)
+  int big_strips;            // phase 1 (one team of all warps) keeps pairs with >= big_strips strips
+  uint2* rb; int64_t rb_cols;   // per CTA: 2 * warps slots (teams x (team_warps + 1) <= 2 * warps)
 };
 
 cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st);

@@ -77,7 +77,7 @@ def test_every_config_both_regimes(menu):
             _assert_equal(out, ref, db, f"menu={menu} m={m} T={T}")
 
 
-@pytest.mark.parametrize("mode", ["team", "t8", "t2", "t1"])
+@pytest.mark.parametrize("mode", ["team", "t8", "t2", "t1", "t2big2", "t1big4"])
 @pytest.mark.parametrize("m", [1, 37, 144, 567, 1500])
 def test_long_sequence_modes(mode, m):
     """Both long-sequence paths (team: strips of query rows; t: transposed, strips of the
@@ -90,7 +90,11 @@ def test_long_sequence_modes(mode, m):
     q = gen.make_query(m, seed=900 + m)
     ref = _oracle(q, BLOSUM62, 10, 2, db)
     for T in (0, 3000):
-        env = {"SW_LONG_MODE": "team"} if mode == "team" else {"SW_LONG_MODE": "t", "SW_T_TEAM": mode[1:]}
+        if mode == "team":
+            env = {"SW_LONG_MODE": "team"}
+        else:   # t<W>[big<S>]: phase-2 team size W, phase-1 (whole CTA) for pairs with >= S strips
+            w, _, big = mode[1:].partition("big")
+            env = {"SW_LONG_MODE": "t", "SW_T_TEAM": w, "SW_T_BIG": big or "1000000"}
         out, st = _gpu(q, BLOSUM62, 10, 2, db, T, env=env)
         _assert_equal(out, ref, db, f"mode={mode} m={m} T={T}")
 
