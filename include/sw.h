@@ -118,6 +118,25 @@ int sw_last_stats(sw_handle h, int64_t out[4]);
  * Milliseconds. */
 int sw_last_kernel_ms(sw_handle h, double out[2]);
 
+/* Optimal local alignment of the handle's query with database sequence seq_index (caller
+ * order) — the traceback step after the search ("The optimal
+ * alignment can be found by backtracking through H").  Computed on the device: an anti-
+ * diagonal sweep of Eq.(1) writing one direction byte per cell (m*n bytes of device scratch),
+ * then a walk back from the first maximal cell.  Query rows [q_begin, q_end) are aligned to
+ * database columns [d_begin, d_end) (0-based, end exclusive; all 0 when score == 0).
+ * ops[0 .. n_ops): runs (length << 2) | op, op 0 = M (q_i against d_j), 1 = I (d_j against a
+ * gap), 2 = D (q_i against a gap); a gap closed and reopened (possible when sigma > rho) is two
+ * runs.  The score of the runs (sum of w over M columns, rho + (len-1)*sigma per gap run)
+ * equals out->score.  If ops_cap < n_ops nothing is copied and SW_E_INVALID is returned with
+ * out->n_ops set.  Blocking. */
+typedef struct {
+  int32_t score;
+  int32_t q_begin, q_end;
+  int32_t d_begin, d_end;
+  int32_t n_ops;
+} sw_alignment;
+int sw_align(sw_handle h, int64_t seq_index, sw_alignment* out, uint32_t* ops, int32_t ops_cap);
+
 /* Free everything (NULL-safe). */
 void sw_destroy(sw_handle h);
 

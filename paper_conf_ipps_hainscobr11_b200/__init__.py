@@ -23,7 +23,7 @@ SW_OK, SW_E_INVALID, SW_E_STATE, SW_E_NOMEM, SW_E_CUDA, SW_E_UNSUPPORTED = range
 SW_AUTO_THRESHOLD = -1
 EXPORTED = ["sw_create", "sw_set_query", "sw_load_db", "sw_search", "sw_search_async",
             "sw_search_batch", "sw_search_batch_async", "sw_last_stats", "sw_last_kernel_ms", "sw_last_threshold",
-            "sw_destroy",
+            "sw_align", "sw_destroy",
             "sw_strerror", "sw_last_error", "sw_version"]
 
 _lib = None
@@ -54,6 +54,8 @@ def load_library(path: str = LIB_PATH):
     L.sw_last_stats.argtypes = [vp, vp]
     L.sw_last_kernel_ms.argtypes = [vp, vp]
     L.sw_last_threshold.argtypes = [vp]
+    L.sw_align.argtypes = [vp, i64, vp, vp, i32]
+    L.sw_align.restype = ctypes.c_int
     L.sw_last_threshold.restype = ctypes.c_int32
     L.sw_destroy.argtypes = [vp]
     L.sw_destroy.restype = None
@@ -155,6 +157,28 @@ def sw_last_kernel_ms(h) -> dict:
     return {"search_ms": float(out[0]), "recompute_ms": float(out[1])}
 
 
+class Alignment(ctypes.Structure):
+    _fields_ = [("score", ctypes.c_int32), ("q_begin", ctypes.c_int32), ("q_end", ctypes.c_int32),
+                ("d_begin", ctypes.c_int32), ("d_end", ctypes.c_int32), ("n_ops", ctypes.c_int32)]
+
+
+OPS = "MID"
+
+
+def sw_align(h, seq_index: int, ops_cap: int = 1 << 16) -> dict:
+    """Optimal local alignment (device traceback) of the handle's query with one sequence."""
+    L = load_library()
+    out = Alignment()
+    ops = np.zeros(max(ops_cap, 1), dtype=np.uint32)
+    st = L.sw_align(h, int(seq_index), ctypes.byref(out), ops.ctypes.data, int(ops_cap))
+    if st != SW_OK and out.n_ops > ops_cap:
+        return sw_align(h, seq_index, int(out.n_ops))
+    _check(h, st)
+    runs = [(OPS[int(v) & 3], int(v) >> 2) for v in ops[: out.n_ops]]
+    return {"score": out.score, "q_begin": out.q_begin, "q_end": out.q_end, "d_begin": out.d_begin,
+            "d_end": out.d_end, "runs": runs, "cigar": "".join(f"{n}{o}" for o, n in runs)}
+
+
 def sw_destroy(h):
     if h:
         load_library().sw_destroy(h)
@@ -188,6 +212,9 @@ class SmithWaterman:
 
     def kernel_ms(self) -> dict:
         return sw_last_kernel_ms(self.h)
+
+    def align(self, seq_index: int) -> dict:
+        return sw_align(self.h, seq_index)
 
     def last_threshold(self) -> int:
         return int(load_library().sw_last_threshold(self.h))

@@ -57,6 +57,14 @@ struct sw_handle_s {
   std::vector<int64_t> sorted_len;     // lengths in sorted (descending) order
   std::vector<int32_t> h_pair_ncols;
   std::vector<int64_t> pair_cols_prefix;  // prefix sums of h_pair_ncols
+  std::vector<int64_t> h_pair_off;        // u16 offset of every pair in d_cols
+  std::vector<int32_t> inv_perm;          // caller index -> sorted position
+  // traceback scratch
+  uint8_t* d_tb_dir = nullptr; size_t tb_dir_cap = 0;
+  int* d_tb_scratch = nullptr; size_t tb_scratch_cap = 0;
+  int* d_tb_result = nullptr; size_t tb_result_cap = 0;
+  uint32_t* d_tb_ops = nullptr; size_t tb_ops_cap = 0;
+  uint8_t* d_tb_query = nullptr; size_t tb_query_cap = 0;
   KernelConfig last_cfg{};
   int32_t last_threshold = 0;
   uint16_t* d_cols = nullptr;
@@ -661,6 +669,9 @@ int sw_load_db(sw_handle h, const uint8_t* residues, int64_t total_residues, con
     pair_off[p + 1] = pair_off[p] + nc + kPadCols;
   }
   const int64_t total_cols = pair_off[n_pairs];
+  h->h_pair_off = pair_off;
+  h->inv_perm.assign((size_t)num_seqs, 0);
+  for (int64_t k = 0; k < num_seqs; ++k) h->inv_perm[perm[k]] = (int32_t)k;
   h->pair_cols_prefix.assign((size_t)n_pairs + 1, 0);
   for (int p = 0; p < n_pairs; ++p) h->pair_cols_prefix[p + 1] = h->pair_cols_prefix[p] + h->h_pair_ncols[p];
   std::vector<uint16_t> cols((size_t)std::max<int64_t>(total_cols, 1));
@@ -766,6 +777,47 @@ int sw_last_stats(sw_handle h, int64_t out[4]) {
 
 int32_t sw_last_threshold(sw_handle h) { return h ? h->last_threshold : -1; }
 
+int sw_align(sw_handle h, int64_t seq_index, sw_alignment* out, uint32_t* ops, int32_t ops_cap) {
+  if (!h) return SW_E_INVALID;
+  if (!h->db_loaded) return fail(h, SW_E_STATE, "sw_load_db has not been called");
+  if (!out || ops_cap < 0 || (ops_cap > 0 && !ops)) return fail(h, SW_E_INVALID, "bad output buffers");
+  if (seq_index < 0 || seq_index >= h->n_seqs) return fail(h, SW_E_INVALID, "seq_index out of range");
+  memset(out, 0, sizeof(*out));
+  const int64_t pos = h->inv_perm[(size_t)seq_index];
+  const int64_t n = h->sorted_len[(size_t)pos];
+  const int m = (int)h->query.size();
+  if (n == 0) { out->q_begin = out->q_end = out->d_begin = out->d_end = 0; return SW_OK; }
+  const int64_t cells = (int64_t)m * n;
+  int rc = grow(h, &h->d_tb_dir, &h->tb_dir_cap, (size_t)cells, "alloc traceback directions");
+  if (rc) return rc;
+  rc = grow(h, &h->d_tb_scratch, &h->tb_scratch_cap, (size_t)7 * m * sizeof(int), "alloc traceback scratch");
+  if (rc) return rc;
+  rc = grow(h, &h->d_tb_result, &h->tb_result_cap, 8 * sizeof(int), "alloc traceback result");
+  if (rc) return rc;
+  const int cap_dev = std::max(1, (int)std::min<int64_t>(m + n, 1 << 24));
+  rc = grow(h, &h->d_tb_ops, &h->tb_ops_cap, (size_t)cap_dev * sizeof(uint32_t), "alloc traceback ops");
+  if (rc) return rc;
+  rc = grow(h, &h->d_tb_query, &h->tb_query_cap, (size_t)m, "alloc traceback query");
+  if (rc) return rc;
+  SW_CUDA(h, cudaMemcpy(h->d_tb_query, h->query.data(), (size_t)m, cudaMemcpyHostToDevice));
+  const int64_t pair = pos >> 1;
+  const int half = (int)(pos & 1);
+  SW_CUDA(h, launch_traceback(h->d_tb_query, m, h->d_cols + h->h_pair_off[(size_t)pair], half, (int)n, h->d_matrix,
+                              h->A, h->rho, h->sigma, h->d_tb_dir, h->d_tb_scratch, h->d_tb_result, h->d_tb_ops,
+                              cap_dev, nullptr));
+  int res[6];
+  SW_CUDA(h, cudaMemcpy(res, h->d_tb_result, sizeof(res), cudaMemcpyDeviceToHost));
+  out->score = res[0];
+  if (res[0] > 0) {
+    out->q_begin = res[3]; out->d_begin = res[4];
+    out->q_end = res[1] + 1; out->d_end = res[2] + 1;
+  }
+  out->n_ops = res[5];
+  if (res[5] > ops_cap) return fail(h, SW_E_INVALID, "ops buffer too small (need " + std::to_string(res[5]) + ")");
+  if (res[5] > 0) SW_CUDA(h, cudaMemcpy(ops, h->d_tb_ops, (size_t)res[5] * sizeof(uint32_t), cudaMemcpyDeviceToHost));
+  return SW_OK;
+}
+
 int sw_last_kernel_ms(sw_handle h, double out[2]) {
   if (!h || !out) return SW_E_INVALID;
   out[0] = out[1] = 0.0;
@@ -795,6 +847,8 @@ void sw_destroy(sw_handle h) {
   }
   cudaFree(h->d_matrix); cudaFree(h->d_cols); cudaFree(h->d_pair_off); cudaFree(h->d_pair_ncols);
   cudaFree(h->d_perm); cudaFree(h->d_scores_tmp); cudaFree(h->d_batch_q);
+  cudaFree(h->d_tb_dir); cudaFree(h->d_tb_scratch); cudaFree(h->d_tb_result); cudaFree(h->d_tb_ops);
+  cudaFree(h->d_tb_query);
   if (h->fork) cudaEventDestroy(h->fork);
   if (h->h_ovf) cudaFreeHost(h->h_ovf);
   delete h;

@@ -119,6 +119,11 @@ cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_
 cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm);
 cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, int pad, cudaStream_t st);
 
+// Traceback of one pair (sw_traceback.cu): dir = m*n bytes, scratch = 7*m ints, result = 6 ints.
+cudaError_t launch_traceback(const uint8_t* q, int m, const uint16_t* dcols, int half, int n, const int8_t* W, int A,
+                             int rho, int sigma, uint8_t* dir, int* scratch, int* result, uint32_t* ops, int ops_cap,
+                             cudaStream_t st);
+
 // Profile image build: byte(rep, a, i) = (i < m && a < A) ? W[q_i][a] + rho : -128.
 cudaError_t launch_profile(uint8_t* blob, const ProfLayout& L, const uint8_t* q, int m, const int8_t* W, int A,
                            int rho, cudaStream_t st);
