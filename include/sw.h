@@ -106,6 +106,23 @@ int sw_search_batch_async(sw_handle h, const uint8_t* queries, const int64_t* q_
 int sw_search_batch(sw_handle h, const uint8_t* queries, const int64_t* q_offsets,
                     int32_t num_queries, int32_t* scores_out, int32_t length_threshold);
 
+/* Streamed database search (extension; §VI: "copy a slice of
+ * the database to the GPU, start aligning, and copy the rest of the database in the
+ * background").  A batch of queries (same form as sw_search_batch; queries == NULL: the
+ * handle's own query, num_queries/q_offsets ignored) against a HOST-resident database (same
+ * CSR form as sw_load_db, only read during the call).  The database is cut into chunks of
+ * whole sequences of about chunk_residues residues; each chunk is sorted and packed on the
+ * host (pinned staging) and copied on an upload stream while the previous chunk is searched,
+ * two device slots alternating (kept on the handle for the next call).  The handle's loaded
+ * database (if any) is neither used nor changed.
+ *   scores_out: HOST int32[num_queries * num_seqs], query-major, caller order.
+ * Blocking.  Errors: as sw_load_db and sw_search_batch; chunk_residues <= 0 -> SW_E_INVALID.
+ * sw_last_stats afterwards sums over the chunks. */
+int sw_search_stream(sw_handle h, const uint8_t* queries, const int64_t* q_offsets, int32_t num_queries,
+                     const uint8_t* residues, int64_t total_residues, const int64_t* offsets,
+                     int64_t num_seqs, int32_t* scores_out, int32_t length_threshold,
+                     int64_t chunk_residues);
+
 /* Statistics of the last search on h (for measurement / tests):
  *   out[0] = number of sequences recomputed in 32-bit after the 16-bit overflow flag,
  *   out[1] = long-path (intra-task) sequences, out[2] = short-path sequences,

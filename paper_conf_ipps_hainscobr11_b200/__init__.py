@@ -22,7 +22,7 @@ LIB_PATH = os.path.join(_HERE, "libsw_b200.so")
 SW_OK, SW_E_INVALID, SW_E_STATE, SW_E_NOMEM, SW_E_CUDA, SW_E_UNSUPPORTED = range(6)
 SW_AUTO_THRESHOLD = -1
 EXPORTED = ["sw_create", "sw_set_query", "sw_load_db", "sw_search", "sw_search_async",
-            "sw_search_batch", "sw_search_batch_async", "sw_last_stats", "sw_last_kernel_ms", "sw_last_threshold",
+            "sw_search_batch", "sw_search_batch_async", "sw_search_stream", "sw_last_stats", "sw_last_kernel_ms", "sw_last_threshold",
             "sw_align", "sw_destroy",
             "sw_strerror", "sw_last_error", "sw_version"]
 
@@ -51,6 +51,7 @@ def load_library(path: str = LIB_PATH):
     L.sw_search_async.argtypes = [vp, vp, i32, vp]
     L.sw_search_batch.argtypes = [vp, vp, vp, i32, vp, i32]
     L.sw_search_batch_async.argtypes = [vp, vp, vp, i32, vp, i32, vp]
+    L.sw_search_stream.argtypes = [vp, vp, vp, i32, vp, i64, vp, i64, vp, i32, i64]
     L.sw_last_stats.argtypes = [vp, vp]
     L.sw_last_kernel_ms.argtypes = [vp, vp]
     L.sw_last_threshold.argtypes = [vp]
@@ -65,7 +66,7 @@ def load_library(path: str = LIB_PATH):
     L.sw_last_error.restype = ctypes.c_char_p
     L.sw_version.restype = ctypes.c_char_p
     for name in ("sw_create", "sw_set_query", "sw_load_db", "sw_search", "sw_search_async", "sw_search_batch",
-                 "sw_search_batch_async", "sw_last_stats", "sw_last_kernel_ms"):
+                 "sw_search_batch_async", "sw_search_stream", "sw_last_stats", "sw_last_kernel_ms"):
         getattr(L, name).restype = ctypes.c_int
     _lib = L
     return L
@@ -144,6 +145,25 @@ def sw_search_batch_async(h, queries, d_scores_ptr: int, length_threshold: int, 
                                                    ctypes.c_void_p(stream_ptr)))
 
 
+def sw_search_stream(h, residues, offsets, length_threshold: int = 3072, chunk_residues: int = 1 << 25,
+                     queries=None) -> np.ndarray:
+    """Search a host-resident database chunk by chunk, uploads overlapped with the search.
+    queries=None: the handle's query, returns int32[num_seqs]; else int32[len(queries), num_seqs]."""
+    r = _u8(residues)
+    off = np.ascontiguousarray(offsets, dtype=np.int64)
+    n = int(off.size - 1)
+    rp = r.ctypes.data if r.size else None
+    if queries is None:
+        qp, op, nq = None, None, 1
+    else:
+        cat, qoff = _batch(queries)
+        qp, op, nq = cat.ctypes.data, qoff.ctypes.data, len(queries)
+    out = np.zeros((nq, max(n, 1)), dtype=np.int32)
+    _check(h, load_library().sw_search_stream(h, qp, op, nq, rp, int(off[-1]), off.ctypes.data, n, out.ctypes.data,
+                                              int(length_threshold), int(chunk_residues)))
+    return out[0, :n] if queries is None else out[:, :n]
+
+
 def sw_last_stats(h) -> dict:
     out = np.zeros(4, dtype=np.int64)
     _check(h, load_library().sw_last_stats(h, out.ctypes.data))
@@ -206,6 +226,10 @@ class SmithWaterman:
 
     def search_batch_into(self, queries, d_scores_ptr: int, length_threshold: int = 3072, stream_ptr: int = 0):
         sw_search_batch_async(self.h, queries, d_scores_ptr, length_threshold, stream_ptr)
+
+    def search_stream(self, residues, offsets, length_threshold: int = 3072, chunk_residues: int = 1 << 25,
+                      queries=None):
+        return sw_search_stream(self.h, residues, offsets, length_threshold, chunk_residues, queries)
 
     def stats(self) -> dict:
         return sw_last_stats(self.h)

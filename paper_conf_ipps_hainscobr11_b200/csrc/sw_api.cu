@@ -9,6 +9,7 @@
 #include <cstring>
 #include <numeric>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "../../include/sw.h"
@@ -41,6 +42,53 @@ struct QuerySlot {
   cudaEvent_t fork = nullptr, join = nullptr;
 };
 
+// One device-resident database in the search layout.
+struct DbState {
+  bool loaded = false;
+  int64_t n_seqs = 0;
+  int n_pairs = 0;
+  std::vector<int64_t> sorted_len;        // lengths in sorted (descending) order
+  std::vector<int32_t> h_pair_ncols;
+  std::vector<int64_t> pair_cols_prefix;  // prefix sums of h_pair_ncols
+  std::vector<int64_t> h_pair_off;        // u16 offset of every pair in d_cols
+  std::vector<int32_t> inv_perm;          // caller index -> sorted position
+  uint16_t* d_cols = nullptr; size_t cols_cap = 0;
+  int64_t* d_pair_off = nullptr; size_t pair_off_cap = 0;
+  int32_t* d_pair_ncols = nullptr; size_t pair_ncols_cap = 0;
+  int32_t* d_perm = nullptr; size_t perm_cap = 0;
+  void* h_stage = nullptr; size_t stage_cap = 0;   // pinned staging for asynchronous uploads
+  void release() {
+    cudaFree(d_cols); cudaFree(d_pair_off); cudaFree(d_pair_ncols); cudaFree(d_perm);
+    if (h_stage) cudaFreeHost(h_stage);
+    d_cols = nullptr; d_pair_off = nullptr; d_pair_ncols = nullptr; d_perm = nullptr; h_stage = nullptr;
+    cols_cap = pair_off_cap = pair_ncols_cap = perm_cap = stage_cap = 0;
+    loaded = false;
+  }
+};
+
+// One of the two alternating chunk slots of sw_search_stream (kept on the handle so repeated
+// streamed searches reuse the pinned staging and device buffers).
+struct StreamSlot {
+  DbState db;
+  cudaStream_t up = nullptr;                 // upload stream
+  cudaEvent_t uploaded = nullptr, searched = nullptr;
+  int32_t* d_sc = nullptr; size_t d_sc_cap = 0;
+  int32_t* h_sc = nullptr; size_t h_sc_cap = 0;   // pinned
+  int32_t* h_ovf = nullptr; int ovf_cap = 0;      // pinned, per query of the chunk
+  int64_t s0 = 0, n = 0;
+  bool pending = false;
+  void release() {
+    if (up) { cudaStreamSynchronize(up); cudaStreamDestroy(up); }
+    if (uploaded) cudaEventDestroy(uploaded);
+    if (searched) { cudaEventSynchronize(searched); cudaEventDestroy(searched); }
+    cudaFree(d_sc);
+    if (h_sc) cudaFreeHost(h_sc);
+    if (h_ovf) cudaFreeHost(h_ovf);
+    db.release();
+    *this = StreamSlot{};
+  }
+};
+
 }  // namespace
 
 struct sw_handle_s {
@@ -50,15 +98,11 @@ struct sw_handle_s {
   int A = 0, rho = 0, sigma = 0, max_w = 0, min_w = 0;
   int8_t* d_matrix = nullptr;
   std::vector<uint8_t> query;
-  // database
-  bool db_loaded = false;
-  int64_t n_seqs = 0;
-  int n_pairs = 0;
-  std::vector<int64_t> sorted_len;     // lengths in sorted (descending) order
-  std::vector<int32_t> h_pair_ncols;
-  std::vector<int64_t> pair_cols_prefix;  // prefix sums of h_pair_ncols
-  std::vector<int64_t> h_pair_off;        // u16 offset of every pair in d_cols
-  std::vector<int32_t> inv_perm;          // caller index -> sorted position
+  // database (the loaded one; sw_search_stream points db at its chunk slots)
+  DbState main_db;
+  DbState* db = &main_db;
+  StreamSlot stream_slot[2];
+  int64_t stat_recomputed = -1;   // >= 0: set by sw_search_stream (sum over its chunks)
   // traceback scratch
   uint8_t* d_tb_dir = nullptr; size_t tb_dir_cap = 0;
   int* d_tb_scratch = nullptr; size_t tb_scratch_cap = 0;
@@ -67,10 +111,6 @@ struct sw_handle_s {
   uint8_t* d_tb_query = nullptr; size_t tb_query_cap = 0;
   KernelConfig last_cfg{};
   int32_t last_threshold = 0;
-  uint16_t* d_cols = nullptr;
-  int64_t* d_pair_off = nullptr;
-  int32_t* d_pair_ncols = nullptr;
-  int32_t* d_perm = nullptr;
   // scratch
   std::vector<QuerySlot> slots;
   int32_t* d_scores_tmp = nullptr;
@@ -280,16 +320,16 @@ int validate_query(sw_handle h, const uint8_t* q, int32_t m) {
 // regime split: sorted_len is descending; long = n >= T (§II-B)
 Split make_split(sw_handle h, int64_t T, int64_t* n_long_seqs_out) {
   const int64_t n_long_seqs =
-      std::lower_bound(h->sorted_len.begin(), h->sorted_len.end(), T, std::greater_equal<int64_t>()) -
-      h->sorted_len.begin();
+      std::lower_bound(h->db->sorted_len.begin(), h->db->sorted_len.end(), T, std::greater_equal<int64_t>()) -
+      h->db->sorted_len.begin();
   const int n_long = (int)((n_long_seqs + 1) / 2);
   Split sp;
   sp.n_long = n_long;
-  sp.n_short = h->n_pairs - n_long;
-  sp.long_cols = h->pair_cols_prefix[n_long];
-  sp.short_cols = h->pair_cols_prefix[h->n_pairs] - sp.long_cols;
-  sp.long_max_cols = n_long ? h->h_pair_ncols[0] : 0;
-  sp.short_max_cols = sp.n_short ? h->h_pair_ncols[n_long] : 0;
+  sp.n_short = h->db->n_pairs - n_long;
+  sp.long_cols = h->db->pair_cols_prefix[n_long];
+  sp.short_cols = h->db->pair_cols_prefix[h->db->n_pairs] - sp.long_cols;
+  sp.long_max_cols = n_long ? h->db->h_pair_ncols[0] : 0;
+  sp.short_max_cols = sp.n_short ? h->db->h_pair_ncols[n_long] : 0;
   if (n_long_seqs_out) *n_long_seqs_out = n_long_seqs;
   return sp;
 }
@@ -303,7 +343,7 @@ Split make_split(sw_handle h, int64_t T, int64_t* n_long_seqs_out) {
 // profiles/r01_sweep_*.jsonl).  Estimated time = max(throughput of both launches,
 // group tail / 0.8); the cheapest candidate wins (ties: the larger T).
 int64_t choose_threshold(sw_handle h, int m) {
-  const int64_t maxlen = h->sorted_len.empty() ? 0 : h->sorted_len[0];
+  const int64_t maxlen = h->db->sorted_len.empty() ? 0 : h->db->sorted_len[0];
   const int64_t cands[] = {maxlen + 1, 16384, 12288, 8192, 6144, 4096, 3072, 2048, 1536, 1024, 768, 512};
   const std::string saved = h->err;
   int64_t chosen = 3072;
@@ -369,13 +409,13 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   const int r_off = (int)round_up(pl.prof_bytes, 256);
   rc = grow(h, &s.d_prof, &s.prof_cap, (size_t)(r_off + pl.r_prof_bytes), "alloc profile", s.stream);
   if (rc) return rc;
-  size_t ovf_bytes = (size_t)std::max<int64_t>(h->n_seqs, 1) * sizeof(int32_t);
+  size_t ovf_bytes = (size_t)std::max<int64_t>(h->db->n_seqs, 1) * sizeof(int32_t);
   size_t ovf_cap = (size_t)s.ovf_cap * sizeof(int32_t);
   rc = grow(h, &s.d_ovf_list, &ovf_cap, ovf_bytes, "alloc overflow list", s.stream);
   if (rc) return rc;
   s.ovf_cap = (int64_t)(ovf_cap / sizeof(int32_t));
-  const int64_t max_cols_all = h->n_pairs ? h->h_pair_ncols[0] + kPadCols : 0;
-  const int64_t max_cols_short = (n_long < h->n_pairs) ? h->h_pair_ncols[n_long] + kPadCols : 0;
+  const int64_t max_cols_all = h->db->n_pairs ? h->db->h_pair_ncols[0] + kPadCols : 0;
+  const int64_t max_cols_short = (n_long < h->db->n_pairs) ? h->db->h_pair_ncols[n_long] + kPadCols : 0;
   const int G = pl.cfg.G;
   size_t rbg = 0;
   if (pl.short_passes > 1 && max_cols_short > 0)
@@ -430,12 +470,12 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   p.rho = h->rho;
   p.sigma = h->sigma;
   p.max_w = h->max_w;
-  p.cols = h->d_cols;
-  p.pair_off = h->d_pair_off;
-  p.pair_ncols = h->d_pair_ncols;
-  p.n_pairs = h->n_pairs;
-  p.n_seqs = (int)h->n_seqs;
-  p.perm = h->d_perm;
+  p.cols = h->db->d_cols;
+  p.pair_off = h->db->d_pair_off;
+  p.pair_ncols = h->db->d_pair_ncols;
+  p.n_pairs = h->db->n_pairs;
+  p.n_seqs = (int)h->db->n_seqs;
+  p.perm = h->db->d_perm;
   p.scores = d_out;
   p.n_long = use_t ? 0 : n_long;
   p.short_begin = n_long;
@@ -468,12 +508,12 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
     t.pad_letter = h->A;
     t.qpair = s.d_qpair;
     t.qcols = qcols;
-    t.cols = h->d_cols;
-    t.pair_off = h->d_pair_off;
-    t.pair_ncols = h->d_pair_ncols;
+    t.cols = h->db->d_cols;
+    t.pair_off = h->db->d_pair_off;
+    t.pair_ncols = h->db->d_pair_ncols;
     t.n_items = n_long;
-    t.n_seqs = (int)h->n_seqs;
-    t.perm = h->d_perm;
+    t.n_seqs = (int)h->db->n_seqs;
+    t.perm = h->db->d_perm;
     t.scores = d_out;
     t.ovf_list = s.d_ovf_list;
     t.ovf_count = s.d_ovf_count;
@@ -515,16 +555,141 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   SW_CUDA(h, cudaMemcpyAsync(h_ovf, s.d_ovf_count, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
 
   h->stat_long += n_long_seqs;
-  h->stat_short += h->n_seqs - n_long_seqs;
+  h->stat_short += h->db->n_seqs - n_long_seqs;
   h->stat_launches += 4 + (pl.lt.off != pl.lg.off ? 1 : 0) + (use_t ? 2 : 0);
+  return SW_OK;
+}
+
+int validate_db(sw_handle h, const uint8_t* residues, int64_t total_residues, const int64_t* offsets,
+                int64_t num_seqs) {
+  if (num_seqs < 0 || total_residues < 0) return fail(h, SW_E_INVALID, "negative size");
+  if (num_seqs > (int64_t)0x7ffffffe) return fail(h, SW_E_INVALID, "num_seqs too large");
+  if (!offsets) return fail(h, SW_E_INVALID, "offsets is NULL");
+  if (total_residues > 0 && !residues) return fail(h, SW_E_INVALID, "residues is NULL");
+  if (offsets[0] != 0 || offsets[num_seqs] != total_residues)
+    return fail(h, SW_E_INVALID, "offsets[0] must be 0 and offsets[num_seqs] == total_residues");
+  for (int64_t k = 0; k < num_seqs; ++k) {
+    const int64_t len = offsets[k + 1] - offsets[k];
+    if (len < 0) return fail(h, SW_E_INVALID, "offsets not non-decreasing at " + std::to_string(k));
+    if (len > SW_MAX_SEQ_LEN) return fail(h, SW_E_INVALID, "sequence longer than SW_MAX_SEQ_LEN at " + std::to_string(k));
+  }
+  uint8_t mx = 0;
+  for (int64_t t = 0; t < total_residues; ++t) mx = std::max(mx, residues[t]);
+  if (mx >= h->A)
+    for (int64_t t = 0; t < total_residues; ++t)
+      if (residues[t] >= h->A) return fail(h, SW_E_INVALID, "residue code >= alphabet_size at " + std::to_string(t));
+  return SW_OK;
+}
+
+// Host preprocessing of a (validated) CSR database into db (§II-C "The database is
+// sorted by length"): stable sort by length descending, pairing, interleaved u16 columns with
+// kPadCols pad columns per pair, upload.  st == nullptr: blocking upload; otherwise the columns
+// are packed into db's pinned staging buffer and copied asynchronously on st (the device
+// buffers are reused when large enough — the caller guarantees they are no longer read).
+int build_db(sw_handle h, DbState& db, const uint8_t* residues, const int64_t* offsets, int64_t num_seqs,
+             cudaStream_t st) {
+  db.loaded = false;
+  std::vector<int64_t> len((size_t)num_seqs);
+  for (int64_t k = 0; k < num_seqs; ++k) len[k] = offsets[k + 1] - offsets[k];
+  std::vector<int32_t> perm((size_t)num_seqs);
+  std::iota(perm.begin(), perm.end(), 0);
+  std::stable_sort(perm.begin(), perm.end(), [&](int32_t a, int32_t b) { return len[a] > len[b]; });
+  db.sorted_len.resize((size_t)num_seqs);
+  for (int64_t k = 0; k < num_seqs; ++k) db.sorted_len[k] = len[perm[k]];
+  const int n_pairs = (int)((num_seqs + 1) / 2);
+  db.h_pair_off.assign((size_t)n_pairs + 1, 0);
+  db.h_pair_ncols.assign((size_t)n_pairs, 0);
+  for (int p = 0; p < n_pairs; ++p) {
+    const int64_t lo = db.sorted_len[2 * p];
+    const int64_t hi = (2 * p + 1 < num_seqs) ? db.sorted_len[2 * p + 1] : 0;
+    const int64_t nc = round_up(std::max<int64_t>({lo, hi, (int64_t)kMinCols}), kColAlign);
+    db.h_pair_ncols[p] = (int32_t)nc;
+    db.h_pair_off[p + 1] = db.h_pair_off[p] + nc + kPadCols;
+  }
+  const int64_t total_cols = db.h_pair_off[n_pairs];
+  db.inv_perm.assign((size_t)num_seqs, 0);
+  for (int64_t k = 0; k < num_seqs; ++k) db.inv_perm[perm[k]] = (int32_t)k;
+  db.pair_cols_prefix.assign((size_t)n_pairs + 1, 0);
+  for (int p = 0; p < n_pairs; ++p) db.pair_cols_prefix[p + 1] = db.pair_cols_prefix[p] + db.h_pair_ncols[p];
+  db.n_seqs = num_seqs;
+  db.n_pairs = n_pairs;
+  const size_t cols_bytes = (size_t)std::max<int64_t>(total_cols, 1) * sizeof(uint16_t);
+  std::vector<uint16_t> cols_vec;
+  uint16_t* cols = nullptr;
+  if (st) {
+    if (db.stage_cap < cols_bytes) {
+      if (db.h_stage) cudaFreeHost(db.h_stage);
+      db.h_stage = nullptr;
+      db.stage_cap = 0;
+      cudaError_t e = cudaMallocHost(&db.h_stage, cols_bytes);
+      if (e != cudaSuccess) return cuda_fail(h, e, "alloc pinned staging");
+      db.stage_cap = cols_bytes;
+    }
+    cols = static_cast<uint16_t*>(db.h_stage);
+  } else {
+    cols_vec.resize(cols_bytes / sizeof(uint16_t));
+    cols = cols_vec.data();
+  }
+  const uint16_t pad = (uint16_t)h->A;
+  auto pack = [&](int p0, int p1) {
+    for (int p = p0; p < p1; ++p) {
+      uint16_t* dst = cols + db.h_pair_off[p];
+      const int64_t nc = db.h_pair_ncols[p];
+      const int64_t s0 = perm[2 * p];
+      const int64_t l0 = len[s0];
+      const uint8_t* r0 = residues ? residues + offsets[s0] : nullptr;
+      const bool has1 = 2 * p + 1 < num_seqs;
+      const int64_t s1 = has1 ? perm[2 * p + 1] : 0;
+      const int64_t l1 = has1 ? len[s1] : 0;
+      const uint8_t* r1 = (has1 && residues) ? residues + offsets[s1] : nullptr;
+      for (int64_t j = 0; j < nc + kPadCols; ++j) {
+        const uint16_t a = j < l0 ? r0[j] : pad;
+        const uint16_t b = j < l1 ? r1[j] : pad;
+        dst[j] = (uint16_t)(a | (b << 8));
+      }
+    }
+  };
+  // packing is host memory bound: split the pairs over a few threads for large databases
+  const int nthreads = n_pairs < (1 << 15) ? 1 : (int)std::min<unsigned>(16u, std::max(1u, std::thread::hardware_concurrency()));
+  if (nthreads == 1) {
+    pack(0, n_pairs);
+  } else {
+    std::vector<std::thread> pool;
+    for (int t = 0; t < nthreads; ++t)
+      pool.emplace_back(pack, (int)((int64_t)n_pairs * t / nthreads), (int)((int64_t)n_pairs * (t + 1) / nthreads));
+    for (auto& t : pool) t.join();
+  }
+  if (num_seqs == 0) { db.loaded = true; return SW_OK; }
+  int rc = grow(h, &db.d_cols, &db.cols_cap, cols_bytes, "alloc database");
+  if (!rc) rc = grow(h, &db.d_pair_off, &db.pair_off_cap, (size_t)n_pairs * sizeof(int64_t), "alloc pair offsets");
+  if (!rc) rc = grow(h, &db.d_pair_ncols, &db.pair_ncols_cap, (size_t)n_pairs * sizeof(int32_t), "alloc pair columns");
+  if (!rc) rc = grow(h, &db.d_perm, &db.perm_cap, (size_t)num_seqs * sizeof(int32_t), "alloc permutation");
+  if (rc) return rc;
+  if (st) {
+    SW_CUDA(h, cudaMemcpyAsync(db.d_cols, cols, cols_bytes, cudaMemcpyHostToDevice, st));
+    // the small index arrays are pageable: their copies complete before returning
+    SW_CUDA(h, cudaMemcpyAsync(db.d_pair_off, db.h_pair_off.data(), (size_t)n_pairs * sizeof(int64_t),
+                               cudaMemcpyHostToDevice, st));
+    SW_CUDA(h, cudaMemcpyAsync(db.d_pair_ncols, db.h_pair_ncols.data(), (size_t)n_pairs * sizeof(int32_t),
+                               cudaMemcpyHostToDevice, st));
+    SW_CUDA(h, cudaMemcpyAsync(db.d_perm, perm.data(), (size_t)num_seqs * sizeof(int32_t), cudaMemcpyHostToDevice, st));
+    SW_CUDA(h, cudaStreamSynchronize(st));   // perm (a local) must outlive its copy
+  } else {
+    SW_CUDA(h, cudaMemcpy(db.d_cols, cols, cols_bytes, cudaMemcpyHostToDevice));
+    SW_CUDA(h, cudaMemcpy(db.d_pair_off, db.h_pair_off.data(), (size_t)n_pairs * sizeof(int64_t), cudaMemcpyHostToDevice));
+    SW_CUDA(h, cudaMemcpy(db.d_pair_ncols, db.h_pair_ncols.data(), (size_t)n_pairs * sizeof(int32_t), cudaMemcpyHostToDevice));
+    SW_CUDA(h, cudaMemcpy(db.d_perm, perm.data(), (size_t)num_seqs * sizeof(int32_t), cudaMemcpyHostToDevice));
+  }
+  db.loaded = true;
   return SW_OK;
 }
 
 int run_batch(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq, int32_t* d_out, int32_t T,
               cudaStream_t user) {
   h->stat_long = h->stat_short = h->stat_launches = 0;
+  h->stat_recomputed = -1;
   h->stat_nq = nq;
-  if (h->n_seqs == 0 || nq == 0) return SW_OK;
+  if (h->db->n_seqs == 0 || nq == 0) return SW_OK;
   // queries run concurrently on up to SW_STREAMS internal streams (default 4) so that the
   // tail of one query's persistent launch overlaps the next query
   int max_streams = 4;
@@ -549,7 +714,7 @@ int run_batch(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq
   for (int k = 0; k < ns; ++k) SW_CUDA(h, cudaStreamWaitEvent(h->slots[k].stream, h->fork, 0));
   for (int k = 0; k < nq; ++k) {
     QuerySlot& s = h->slots[k % ns];
-    rc = enqueue_query(h, s, d_queries + qoff[k], (int)(qoff[k + 1] - qoff[k]), d_out + (int64_t)k * h->n_seqs, T,
+    rc = enqueue_query(h, s, d_queries + qoff[k], (int)(qoff[k + 1] - qoff[k]), d_out + (int64_t)k * h->db->n_seqs, T,
                        h->h_ovf + k, h->ev.data() + 3 * k);
     if (rc) return rc;
   }
@@ -632,89 +797,157 @@ int sw_set_query(sw_handle h, const uint8_t* query, int32_t query_len) {
 int sw_load_db(sw_handle h, const uint8_t* residues, int64_t total_residues, const int64_t* offsets,
                int64_t num_seqs) {
   if (!h) return SW_E_INVALID;
-  if (num_seqs < 0 || total_residues < 0) return fail(h, SW_E_INVALID, "negative size");
-  if (num_seqs > (int64_t)0x7ffffffe) return fail(h, SW_E_INVALID, "num_seqs too large");
-  if (!offsets) return fail(h, SW_E_INVALID, "offsets is NULL");
-  if (total_residues > 0 && !residues) return fail(h, SW_E_INVALID, "residues is NULL");
-  if (offsets[0] != 0 || offsets[num_seqs] != total_residues)
-    return fail(h, SW_E_INVALID, "offsets[0] must be 0 and offsets[num_seqs] == total_residues");
-  std::vector<int64_t> len((size_t)num_seqs);
-  for (int64_t k = 0; k < num_seqs; ++k) {
-    len[k] = offsets[k + 1] - offsets[k];
-    if (len[k] < 0) return fail(h, SW_E_INVALID, "offsets not non-decreasing at " + std::to_string(k));
-    if (len[k] > SW_MAX_SEQ_LEN) return fail(h, SW_E_INVALID, "sequence longer than SW_MAX_SEQ_LEN at " + std::to_string(k));
-  }
-  for (int64_t t = 0; t < total_residues; ++t)
-    if (residues[t] >= h->A) return fail(h, SW_E_INVALID, "residue code >= alphabet_size at " + std::to_string(t));
+  int rc = validate_db(h, residues, total_residues, offsets, num_seqs);
+  if (rc) return rc;
+  h->db = &h->main_db;
+  h->main_db.release();
+  return build_db(h, h->main_db, residues, offsets, num_seqs, nullptr);
+}
 
-  // free the previous database
-  cudaFree(h->d_cols); cudaFree(h->d_pair_off); cudaFree(h->d_pair_ncols); cudaFree(h->d_perm);
-  h->d_cols = nullptr; h->d_pair_off = nullptr; h->d_pair_ncols = nullptr; h->d_perm = nullptr;
-  h->db_loaded = false;
-
-  // stable sort by length, descending (ties keep input order)
-  std::vector<int32_t> perm((size_t)num_seqs);
-  std::iota(perm.begin(), perm.end(), 0);
-  std::stable_sort(perm.begin(), perm.end(), [&](int32_t a, int32_t b) { return len[a] > len[b]; });
-  h->sorted_len.resize((size_t)num_seqs);
-  for (int64_t k = 0; k < num_seqs; ++k) h->sorted_len[k] = len[perm[k]];
-  const int n_pairs = (int)((num_seqs + 1) / 2);
-  std::vector<int64_t> pair_off((size_t)n_pairs + 1, 0);
-  h->h_pair_ncols.assign((size_t)n_pairs, 0);
-  for (int p = 0; p < n_pairs; ++p) {
-    const int64_t lo = h->sorted_len[2 * p];
-    const int64_t hi = (2 * p + 1 < num_seqs) ? h->sorted_len[2 * p + 1] : 0;
-    const int64_t nc = round_up(std::max<int64_t>({lo, hi, (int64_t)kMinCols}), kColAlign);
-    h->h_pair_ncols[p] = (int32_t)nc;
-    pair_off[p + 1] = pair_off[p] + nc + kPadCols;
+int sw_search_stream(sw_handle h, const uint8_t* queries, const int64_t* q_offsets, int32_t num_queries,
+                     const uint8_t* residues, int64_t total_residues, const int64_t* offsets, int64_t num_seqs,
+                     int32_t* scores_out, int32_t length_threshold, int64_t chunk_residues) {
+  if (!h) return SW_E_INVALID;
+  int64_t own_qo[2] = {0, (int64_t)h->query.size()};
+  if (!queries) {                       // the handle's own query
+    queries = h->query.data();
+    q_offsets = own_qo;
+    num_queries = 1;
   }
-  const int64_t total_cols = pair_off[n_pairs];
-  h->h_pair_off = pair_off;
-  h->inv_perm.assign((size_t)num_seqs, 0);
-  for (int64_t k = 0; k < num_seqs; ++k) h->inv_perm[perm[k]] = (int32_t)k;
-  h->pair_cols_prefix.assign((size_t)n_pairs + 1, 0);
-  for (int p = 0; p < n_pairs; ++p) h->pair_cols_prefix[p + 1] = h->pair_cols_prefix[p] + h->h_pair_ncols[p];
-  std::vector<uint16_t> cols((size_t)std::max<int64_t>(total_cols, 1));
-  const uint16_t pad = (uint16_t)h->A;
-  for (int p = 0; p < n_pairs; ++p) {
-    uint16_t* dst = cols.data() + pair_off[p];
-    const int64_t nc = h->h_pair_ncols[p];
-    const int64_t s0 = perm[2 * p];
-    const int64_t l0 = len[s0];
-    const uint8_t* r0 = residues ? residues + offsets[s0] : nullptr;
-    const bool has1 = 2 * p + 1 < num_seqs;
-    const int64_t s1 = has1 ? perm[2 * p + 1] : 0;
-    const int64_t l1 = has1 ? len[s1] : 0;
-    const uint8_t* r1 = (has1 && residues) ? residues + offsets[s1] : nullptr;
-    for (int64_t j = 0; j < nc + kPadCols; ++j) {
-      const uint16_t a = j < l0 ? r0[j] : pad;
-      const uint16_t b = j < l1 ? r1[j] : pad;
-      dst[j] = (uint16_t)(a | (b << 8));
+  if (num_queries < 0 || !q_offsets) return fail(h, SW_E_INVALID, "bad query batch");
+  if (q_offsets[0] != 0) return fail(h, SW_E_INVALID, "q_offsets[0] != 0");
+  for (int k = 0; k < num_queries; ++k) {
+    const int64_t m = q_offsets[k + 1] - q_offsets[k];
+    if (m <= 0 || m > SW_MAX_QUERY_LEN) return fail(h, SW_E_INVALID, "query length out of range in batch");
+    int rc = validate_query(h, queries + q_offsets[k], (int32_t)m);
+    if (rc) return rc;
+  }
+  if (num_seqs > 0 && num_queries > 0 && !scores_out) return fail(h, SW_E_INVALID, "scores_out is NULL");
+  if (chunk_residues <= 0) return fail(h, SW_E_INVALID, "chunk_residues <= 0");
+  if (length_threshold < 0 && length_threshold != SW_AUTO_THRESHOLD)
+    return fail(h, SW_E_INVALID, "length_threshold < 0 (use SW_AUTO_THRESHOLD for automatic)");
+  int rc = validate_db(h, residues, total_residues, offsets, num_seqs);
+  if (rc) return rc;
+  h->stat_long = h->stat_short = h->stat_launches = 0;
+  h->stat_recomputed = 0;
+  if (num_seqs == 0 || num_queries == 0) return SW_OK;
+  rc = ensure_slots(h, 1);
+  if (rc) return rc;
+  cudaStream_t st = h->slots[0].stream;
+  const int nq = num_queries;
+  const int64_t qtot = q_offsets[nq];
+  size_t qcap = (size_t)h->batch_q_cap;
+  rc = grow(h, &h->d_batch_q, &qcap, (size_t)qtot, "alloc stream queries", st);
+  if (rc) return rc;
+  h->batch_q_cap = (int64_t)qcap;
+  std::vector<int64_t> qo(q_offsets, q_offsets + nq + 1);
+  SW_CUDA(h, cudaMemcpyAsync(h->d_batch_q, queries, (size_t)qtot, cudaMemcpyHostToDevice, st));
+  SW_CUDA(h, cudaStreamSynchronize(st));     // the caller's query buffer is pageable
+  // chunk boundaries: whole sequences, about chunk_residues residues each
+  std::vector<int64_t> cut{0};
+  while (cut.back() < num_seqs) {
+    const int64_t s0 = cut.back();
+    int64_t e = std::upper_bound(offsets + s0, offsets + num_seqs + 1, offsets[s0] + chunk_residues) - offsets - 1;
+    cut.push_back(std::min(std::max(e, s0 + 1), num_seqs));
+  }
+  const int nchunks = (int)cut.size() - 1;
+  for (auto& ss : h->stream_slot) {
+    if (!ss.up && cudaStreamCreateWithFlags(&ss.up, cudaStreamNonBlocking) != cudaSuccess)
+      return fail(h, SW_E_CUDA, "stream setup");
+    if (!ss.uploaded && cudaEventCreateWithFlags(&ss.uploaded, cudaEventDisableTiming) != cudaSuccess)
+      return fail(h, SW_E_CUDA, "stream setup");
+    if (!ss.searched && cudaEventCreateWithFlags(&ss.searched, cudaEventDisableTiming) != cudaSuccess)
+      return fail(h, SW_E_CUDA, "stream setup");
+    ss.pending = false;
+  }
+  int64_t stat_long = 0, stat_short = 0, stat_launches = 0, stat_rec = 0;
+  // wait for slot k's search; hand its scores over
+  auto finish = [&](StreamSlot& ss) -> int {
+    if (!ss.pending) return SW_OK;
+    ss.pending = false;
+    cudaError_t e = cudaEventSynchronize(ss.searched);
+    if (e != cudaSuccess) return cuda_fail(h, e, "streamed chunk search");
+    for (int q = 0; q < nq; ++q) {
+      memcpy(scores_out + (int64_t)q * num_seqs + ss.s0, ss.h_sc + (int64_t)q * ss.n, (size_t)ss.n * sizeof(int32_t));
+      stat_rec += ss.h_ovf[q];
     }
+    return SW_OK;
+  };
+  // run_batch keeps its overflow counts in h->h_ovf: point it at the chunk slot's array
+  int32_t* const saved_ovf = h->h_ovf;
+  const int saved_ovf_cap = h->h_ovf_cap;
+  for (int c = 0; c < nchunks && rc == SW_OK; ++c) {
+    StreamSlot& ss = h->stream_slot[c & 1];
+    rc = finish(ss);                     // slot's previous chunk must be done before reuse
+    if (rc) break;
+    const int64_t s0 = cut[c], s1 = cut[c + 1], n = s1 - s0;
+    std::vector<int64_t> off((size_t)n + 1);
+    for (int64_t i = 0; i <= n; ++i) off[i] = offsets[s0 + i] - offsets[s0];
+    // host packing + upload of chunk c overlap the device search of chunk c - 1
+    // ("copy a slice of the database to the GPU, start aligning, and copy the rest of the
+    // database in the background", §VI)
+    rc = build_db(h, ss.db, residues + offsets[s0], off.data(), n, ss.up);
+    if (rc) break;
+    const size_t need = (size_t)nq * (size_t)n * sizeof(int32_t);
+    if (ss.d_sc_cap < need) {
+      cudaFree(ss.d_sc);
+      ss.d_sc = nullptr; ss.d_sc_cap = 0;
+      if (cudaMalloc(&ss.d_sc, need) != cudaSuccess) { rc = fail(h, SW_E_NOMEM, "stream score buffer"); break; }
+      ss.d_sc_cap = need;
+    }
+    if (ss.h_sc_cap < need) {
+      if (ss.h_sc) cudaFreeHost(ss.h_sc);
+      ss.h_sc = nullptr; ss.h_sc_cap = 0;
+      if (cudaMallocHost(&ss.h_sc, need) != cudaSuccess) { rc = fail(h, SW_E_NOMEM, "stream score buffer"); break; }
+      ss.h_sc_cap = need;
+    }
+    if (ss.ovf_cap < nq) {
+      if (ss.h_ovf) cudaFreeHost(ss.h_ovf);
+      ss.h_ovf = nullptr; ss.ovf_cap = 0;
+      if (cudaMallocHost(&ss.h_ovf, (size_t)nq * sizeof(int32_t)) != cudaSuccess) {
+        rc = fail(h, SW_E_NOMEM, "stream overflow counts");
+        break;
+      }
+      ss.ovf_cap = nq;
+    }
+    if (cudaEventRecord(ss.uploaded, ss.up) != cudaSuccess || cudaStreamWaitEvent(st, ss.uploaded, 0) != cudaSuccess) {
+      rc = fail(h, SW_E_CUDA, "stream event");
+      break;
+    }
+    h->db = &ss.db;
+    h->h_ovf = ss.h_ovf;
+    h->h_ovf_cap = ss.ovf_cap;
+    rc = run_batch(h, h->d_batch_q, qo.data(), nq, ss.d_sc, length_threshold, st);
+    h->db = &h->main_db;
+    if (rc) break;
+    stat_long += h->stat_long; stat_short += h->stat_short; stat_launches += h->stat_launches;
+    if (cudaMemcpyAsync(ss.h_sc, ss.d_sc, need, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+        cudaEventRecord(ss.searched, st) != cudaSuccess) {
+      rc = fail(h, SW_E_CUDA, "stream score copy");
+      break;
+    }
+    ss.s0 = s0; ss.n = n; ss.pending = true;
   }
-  h->n_seqs = num_seqs;
-  h->n_pairs = n_pairs;
-  if (num_seqs == 0) { h->db_loaded = true; return SW_OK; }
-  SW_CUDA(h, cudaMalloc(&h->d_cols, cols.size() * sizeof(uint16_t)));
-  SW_CUDA(h, cudaMalloc(&h->d_pair_off, (size_t)n_pairs * sizeof(int64_t)));
-  SW_CUDA(h, cudaMalloc(&h->d_pair_ncols, (size_t)n_pairs * sizeof(int32_t)));
-  SW_CUDA(h, cudaMalloc(&h->d_perm, (size_t)num_seqs * sizeof(int32_t)));
-  SW_CUDA(h, cudaMemcpy(h->d_cols, cols.data(), cols.size() * sizeof(uint16_t), cudaMemcpyHostToDevice));
-  SW_CUDA(h, cudaMemcpy(h->d_pair_off, pair_off.data(), (size_t)n_pairs * sizeof(int64_t), cudaMemcpyHostToDevice));
-  SW_CUDA(h, cudaMemcpy(h->d_pair_ncols, h->h_pair_ncols.data(), (size_t)n_pairs * sizeof(int32_t), cudaMemcpyHostToDevice));
-  SW_CUDA(h, cudaMemcpy(h->d_perm, perm.data(), (size_t)num_seqs * sizeof(int32_t), cudaMemcpyHostToDevice));
-  h->db_loaded = true;
-  return SW_OK;
+  for (auto& ss : h->stream_slot) {
+    const int r2 = finish(ss);
+    if (rc == SW_OK) rc = r2;
+  }
+  h->db = &h->main_db;
+  h->h_ovf = saved_ovf;
+  h->h_ovf_cap = saved_ovf_cap;
+  h->stat_long = stat_long; h->stat_short = stat_short; h->stat_launches = stat_launches;
+  h->stat_recomputed = stat_rec;
+  return rc;
 }
 
 int sw_search_batch_async(sw_handle h, const uint8_t* queries, const int64_t* q_offsets, int32_t num_queries,
                           int32_t* d_scores_out, int32_t length_threshold, void* cuda_stream) {
   if (!h) return SW_E_INVALID;
-  if (!h->db_loaded) return fail(h, SW_E_STATE, "sw_load_db has not been called");
+  if (!h->db->loaded) return fail(h, SW_E_STATE, "sw_load_db has not been called");
   if (num_queries < 0 || !q_offsets || (num_queries > 0 && !queries)) return fail(h, SW_E_INVALID, "bad query batch");
   if (length_threshold < 0 && length_threshold != SW_AUTO_THRESHOLD)
     return fail(h, SW_E_INVALID, "length_threshold < 0 (use SW_AUTO_THRESHOLD for automatic)");
-  if (h->n_seqs > 0 && num_queries > 0 && !d_scores_out) return fail(h, SW_E_INVALID, "d_scores_out is NULL");
+  if (h->db->n_seqs > 0 && num_queries > 0 && !d_scores_out) return fail(h, SW_E_INVALID, "d_scores_out is NULL");
   if (q_offsets[0] != 0) return fail(h, SW_E_INVALID, "q_offsets[0] != 0");
   for (int k = 0; k < num_queries; ++k) {
     const int64_t m = q_offsets[k + 1] - q_offsets[k];
@@ -741,9 +974,9 @@ int sw_search_async(sw_handle h, int32_t* d_scores_out, int32_t length_threshold
 int sw_search_batch(sw_handle h, const uint8_t* queries, const int64_t* q_offsets, int32_t num_queries,
                     int32_t* scores_out, int32_t length_threshold) {
   if (!h) return SW_E_INVALID;
-  if (!h->db_loaded) return fail(h, SW_E_STATE, "sw_load_db has not been called");
+  if (!h->db->loaded) return fail(h, SW_E_STATE, "sw_load_db has not been called");
   if (num_queries < 0) return fail(h, SW_E_INVALID, "num_queries < 0");
-  const int64_t need = (int64_t)num_queries * h->n_seqs;
+  const int64_t need = (int64_t)num_queries * h->db->n_seqs;
   if (need > 0 && !scores_out) return fail(h, SW_E_INVALID, "scores_out is NULL");
   size_t cap = (size_t)h->scores_tmp_cap * sizeof(int32_t);
   int rc = grow(h, &h->d_scores_tmp, &cap, (size_t)std::max<int64_t>(need, 1) * sizeof(int32_t), "alloc scores");
@@ -768,7 +1001,7 @@ int sw_last_stats(sw_handle h, int64_t out[4]) {
   int64_t ovf = 0;
   // valid once the last search's stream work has completed
   for (int k = 0; k < std::min(h->stat_nq, h->h_ovf_cap); ++k) ovf += h->h_ovf[k];
-  out[0] = ovf;
+  out[0] = h->stat_recomputed >= 0 ? h->stat_recomputed : ovf;
   out[1] = h->stat_long;
   out[2] = h->stat_short;
   out[3] = h->stat_launches;
@@ -779,12 +1012,12 @@ int32_t sw_last_threshold(sw_handle h) { return h ? h->last_threshold : -1; }
 
 int sw_align(sw_handle h, int64_t seq_index, sw_alignment* out, uint32_t* ops, int32_t ops_cap) {
   if (!h) return SW_E_INVALID;
-  if (!h->db_loaded) return fail(h, SW_E_STATE, "sw_load_db has not been called");
+  if (!h->db->loaded) return fail(h, SW_E_STATE, "sw_load_db has not been called");
   if (!out || ops_cap < 0 || (ops_cap > 0 && !ops)) return fail(h, SW_E_INVALID, "bad output buffers");
-  if (seq_index < 0 || seq_index >= h->n_seqs) return fail(h, SW_E_INVALID, "seq_index out of range");
+  if (seq_index < 0 || seq_index >= h->db->n_seqs) return fail(h, SW_E_INVALID, "seq_index out of range");
   memset(out, 0, sizeof(*out));
-  const int64_t pos = h->inv_perm[(size_t)seq_index];
-  const int64_t n = h->sorted_len[(size_t)pos];
+  const int64_t pos = h->db->inv_perm[(size_t)seq_index];
+  const int64_t n = h->db->sorted_len[(size_t)pos];
   const int m = (int)h->query.size();
   if (n == 0) { out->q_begin = out->q_end = out->d_begin = out->d_end = 0; return SW_OK; }
   const int64_t cells = (int64_t)m * n;
@@ -802,7 +1035,7 @@ int sw_align(sw_handle h, int64_t seq_index, sw_alignment* out, uint32_t* ops, i
   SW_CUDA(h, cudaMemcpy(h->d_tb_query, h->query.data(), (size_t)m, cudaMemcpyHostToDevice));
   const int64_t pair = pos >> 1;
   const int half = (int)(pos & 1);
-  SW_CUDA(h, launch_traceback(h->d_tb_query, m, h->d_cols + h->h_pair_off[(size_t)pair], half, (int)n, h->d_matrix,
+  SW_CUDA(h, launch_traceback(h->d_tb_query, m, h->db->d_cols + h->db->h_pair_off[(size_t)pair], half, (int)n, h->d_matrix,
                               h->A, h->rho, h->sigma, h->d_tb_dir, h->d_tb_scratch, h->d_tb_result, h->d_tb_ops,
                               cap_dev, nullptr));
   int res[6];
@@ -845,8 +1078,10 @@ void sw_destroy(sw_handle h) {
     if (s.join) cudaEventDestroy(s.join);
     if (s.done) cudaEventDestroy(s.done);
   }
-  cudaFree(h->d_matrix); cudaFree(h->d_cols); cudaFree(h->d_pair_off); cudaFree(h->d_pair_ncols);
-  cudaFree(h->d_perm); cudaFree(h->d_scores_tmp); cudaFree(h->d_batch_q);
+  cudaFree(h->d_matrix);
+  h->main_db.release();
+  for (auto& ss : h->stream_slot) ss.release();
+  cudaFree(h->d_scores_tmp); cudaFree(h->d_batch_q);
   cudaFree(h->d_tb_dir); cudaFree(h->d_tb_scratch); cudaFree(h->d_tb_result); cudaFree(h->d_tb_ops);
   cudaFree(h->d_tb_query);
   if (h->fork) cudaEventDestroy(h->fork);

@@ -117,3 +117,47 @@ def test_version_and_null_destroy():
     L = swp.load_library()
     assert L.sw_version().startswith(b"sw_b200")
     L.sw_destroy(ctypes.c_void_p())
+
+
+@pytest.mark.parametrize("chunk", [1, 997, 20000, 1 << 30])
+def test_search_stream_matches_oracle(chunk):
+    """sw_search_stream (f3): chunked, upload-overlapped search == oracle for any chunk size,
+    including one sequence per chunk and a single chunk; the loaded database is untouched."""
+    db = gen.build_database(np.concatenate([gen.sp_lengths(900, seed=12), [4000, 0, 3500, 1]]), 12)
+    q = gen.make_query(222)
+    ref = oracle.scores(q, BLOSUM62, 10, 2, db.residues, db.offsets)
+    other = _db(30, seed=2)
+    with swp.SmithWaterman(q, BLOSUM62, 10, 2) as sw:
+        sw.load_db(other.residues, other.offsets)
+        out = sw.search_stream(db.residues, db.offsets, 3072 if chunk != 997 else swp.SW_AUTO_THRESHOLD, chunk)
+        assert np.array_equal(out, ref)
+        assert sw.stats()["long_seqs"] + sw.stats()["short_seqs"] == db.num_seqs
+        assert np.array_equal(sw.search(3072), oracle.scores(q, BLOSUM62, 10, 2, other.residues, other.offsets))
+        qs = [gen.make_query(L) for L in (7, 300, 1200)]
+        outb = sw.search_stream(db.residues, db.offsets, 3072, chunk, queries=qs)
+        for k, qq in enumerate(qs):
+            assert np.array_equal(outb[k], oracle.scores(qq, BLOSUM62, 10, 2, db.residues, db.offsets))
+
+
+def test_search_stream_errors_and_empty():
+    L = swp.load_library()
+    with swp.SmithWaterman(gen.make_query(40), BLOSUM62, 10, 2) as sw:
+        out = sw.search_stream(np.zeros(0, np.uint8), np.array([0], np.int64))
+        assert out.shape == (0,)
+        res = np.zeros(10, np.uint8)
+        off = np.array([0, 10], np.int64)
+        sc = np.zeros(1, np.int32)
+        def call(roff=off, out=sc, chunk=64, qs=None, qo=None, nq=1):
+            return L.sw_search_stream(sw.h, qs, qo, nq, res.ctypes.data, 10, roff.ctypes.data, 1, out, 3072, chunk)
+        assert call(out=sc.ctypes.data, chunk=0) == swp.SW_E_INVALID
+        assert call(roff=np.array([0, 11], np.int64), out=sc.ctypes.data) == swp.SW_E_INVALID
+        assert call(out=None) == swp.SW_E_INVALID
+        badq, qo = np.array([1, 40], np.uint8), np.array([0, 2], np.int64)
+        assert call(out=sc.ctypes.data, qs=badq.ctypes.data, qo=qo.ctypes.data) == swp.SW_E_INVALID
+        assert call(out=sc.ctypes.data) == swp.SW_OK and sc[0] == oracle.scores(
+            gen.make_query(40), BLOSUM62, 10, 2, res, off)[0]
+        # overflow counts are summed over chunks
+        hp = np.full(3000, 17, np.uint8)              # W-W = 11: 33000 > int16
+        sw.set_query(hp)
+        out = sw.search_stream(np.concatenate([hp, hp]), np.array([0, 3000, 6000], np.int64), 3072, 3000)
+        assert list(out) == [3000 * int(BLOSUM62[17, 17])] * 2 and sw.stats()["recomputed_s32"] == 2
