@@ -162,6 +162,13 @@ int grow(sw_handle h, T** p, size_t* cap, size_t bytes, const char* what, cudaSt
 
 int64_t round_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
 
+// G = 32 group items run as one continuous stream per warp (sw_engine.cuh group_stream);
+// SW_GROUP_STREAM=0 selects the per-strip sweeps instead (A/B measurements, tests)
+bool group_stream_enabled() {
+  const char* f = getenv("SW_GROUP_STREAM");
+  return !(f && f[0] == '0');
+}
+
 // ------------------------------------------------------------------------------------ planning
 ProfLayout make_layout(int off, int G, int R, int m, int A1, int nrep) {
   ProfLayout L;
@@ -246,7 +253,9 @@ int make_plan(sw_handle h, int m, const Split& sp, Plan* pl) {
     const double lat = 1.0 - 0.025 * std::min(2.0, std::max(0.0, wps - 2.0));
     const double is = (6.5 * c.Rs + 24.0) * lat, il = (6.5 * c.Rl + 40.0) * lat;
     const int W = team_warps_for(lt.strips, c.threads / 32);
-    const double gsteps = ((double)sp.short_cols + (double)sp.n_short * (c.G - 1)) * lg.strips / (32 / c.G);
+    // (G = 32 streams: a 4-column gap per segment plus ~3 steps' worth of per-lane resets)
+    const double fill = (c.G == 32 && group_stream_enabled()) ? 7.0 : c.G - 1.0;
+    const double gsteps = ((double)sp.short_cols + (double)sp.n_short * fill) * lg.strips / (32 / c.G);
     const double tsteps = ((double)sp.long_cols + 31.0 * sp.n_long) * lt.strips;
     double thr = (gsteps * is + tsteps * il) / kGpuIssue;
     // few items: the issue rate needs ~2 busy warps per scheduler (4 per SM)
@@ -302,7 +311,9 @@ int ensure_slots(sw_handle h, int n) {
     SW_CUDA(h, cudaEventCreateWithFlags(&s.fork, cudaEventDisableTiming));
     SW_CUDA(h, cudaEventCreateWithFlags(&s.join, cudaEventDisableTiming));
     SW_CUDA(h, cudaEventCreateWithFlags(&s.done, cudaEventDisableTiming));
-    SW_CUDA(h, cudaMalloc(&s.d_work, 4 * sizeof(int32_t)));
+    // 4 work counters, then 4 neutral row-buffer entries (uint2 zeros) read by group_stream
+    SW_CUDA(h, cudaMalloc(&s.d_work, 12 * sizeof(int32_t)));
+    SW_CUDA(h, cudaMemset(s.d_work, 0, 12 * sizeof(int32_t)));
     SW_CUDA(h, cudaMalloc(&s.d_ovf_count, sizeof(int32_t)));
     h->slots.push_back(s);
   }
@@ -482,6 +493,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   p.item_list = nullptr;
   p.item_count = nullptr;
   p.work = s.d_work;
+  p.rb_zero = reinterpret_cast<const uint2*>(s.d_work + 4);
   p.ovf_list = s.d_ovf_list;
   p.ovf_count = s.d_ovf_count;
   p.short_passes = pl.short_passes;
@@ -489,6 +501,8 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   p.team_warps = pl.team_warps;
   p.rb_group = s.d_rb_group;
   p.rb_group_cols = max_cols_short;
+  // (the stream addresses columns with 32-bit indices)
+  p.group_stream = group_stream_enabled() && h->db->h_pair_off[h->db->n_pairs] < (int64_t)INT32_MAX;
   p.rb_team = s.d_rb_team;
   p.rb_team_cols = max_cols_all;
   SW_CUDA(h, cudaEventRecord(ev[0], st));

@@ -346,6 +346,208 @@ __device__ __forceinline__ void emit(const SearchParams& p, uint32_t b, int pair
   }
 }
 
+// Continuous group stream for whole-warp chains (G = 32, one pair per chain).  run_pass
+// gives every (pair, strip) its own sweep: the chain fills for 31 steps and drains for 31 more,
+// ~8 % of the lane-steps at Swiss-Prot lengths.  Here the strips and pairs a warp takes form
+// ONE column stream (§VI: process the strips "in a single pass ... the pipeline
+// only has to be filled and flushed once"): lane l processes stream position t - l at step t,
+// so lane 0 starts the next segment (strip or pair) while the other lanes still finish the
+// previous one.  Every segment starts with a gap of 4 pad positions (segment lengths are
+// multiples of 4, so the gap is exactly the fetch set of one 4-step group); a lane moves into
+// the next segment (resets its rows to the neutral state, c4) at the 4-step group boundary that
+// falls inside its gap window, so the 4-step body stays branch-free.  In the gap:
+//  * a lane that already switched sees pad letters and neutral vertical input (below), stays
+//    exactly neutral and reaches the real columns in the neutral state;
+//  * a lane that has not switched yet ("stale") computes pad cells from its old state; their H
+//    cannot exceed the old segment's maximum (a pad column only adds -128 or gap costs);
+//  * resets happen only at group boundaries and a lane's gap window starts one step after the
+//    lane above's, so a switched lane can receive a stale value only at the boundary where both
+//    switch, from the upper lane's last step: that lane neutralises its outgoing (H, F + rho)
+//    as it switches.
+// Segments are >= kMinCols + 4 = 52 positions, so at most two are in flight, and the strip
+// hand-off is ordered: lane 31 writes row-buffer column j at step T + 4 + 31 + j, lane 0
+// fetches it for the next strip at step T + len + 4 + j >= T + 52 + j (__syncwarp every group
+// in between).  A pair's score is reduced across the lanes once its last lane has moved on
+// (each lane parks its maximum in bdone when it leaves the pair's last strip).
+template <class L, int R, bool PP>
+__device__ __forceinline__ void group_stream(const SearchParams& p, const ChainConst& c, const uint8_t* pbase,
+                                             uint2* __restrict__ rb) {
+  static_assert(R % 4 == 0, "R must be a multiple of 4");
+  constexpr int kGap = 4;
+  const int lane = threadIdx.x & 31;
+  const uint32_t nrho = L::splat(-c.rho);
+  const uint32_t nsig = L::splat(-c.sigma);
+  constexpr int CB = chunk_bytes<R>();
+  constexpr int kStripBytes = R * 32;          // (R / CB) chunks x 32 lanes x CB bytes
+  constexpr int kEndLen = 0xffffff;            // the END segment (after the last pair) never ends
+  const int passes = p.short_passes;
+  const int nshort = p.n_pairs - p.short_begin;
+  const int ls = p.lg.ls;
+
+  // ---- warp-uniform fetch cursor: lane 0's stream, one group (4 positions) ahead of lane 0
+  auto take = [&]() -> int {
+    int b = 0;
+    if (lane == 0) b = atomicAdd(&p.work[1], 1);
+    return __shfl_sync(SWB_FULL, b, 0);
+  };
+  int nx_pair = -1, nx_len = kEndLen;
+  int64_t nx_off = 0;
+  auto prefetch = [&]() {   // next pair of the queue (its header loads overlap the current pair)
+    const int item = take();
+    if (item < nshort) {
+      nx_pair = p.short_begin + item;
+      nx_off = p.pair_off[nx_pair];
+      nx_len = p.pair_ncols[nx_pair] + kGap;
+    } else {
+      nx_pair = -1; nx_len = kEndLen;
+    }
+  };
+  prefetch();
+  if (nx_pair < 0) return;
+  int f_pair = nx_pair, f_len = nx_len, f_P = 0, f_col = 0;
+  const uint16_t* f_cols = p.cols + nx_off;
+  const uint16_t* f_pad = f_cols + (f_len - kGap);   // the pair's trailing pad columns
+  nx_pair = -2;                                   // -2: the next pair is not fetched yet
+  if (passes == 1) prefetch();
+  // descriptors (len | (P + 1) << 24) of the two newest segments, by segment parity
+  uint32_t desc0 = (uint32_t)f_len | (1u << 24), desc1 = 0;
+  int f_seg = 0;
+  int fn = 0;                 // index of the next fetch (= the step at which lane 0 consumes it)
+  bool pending = false;       // a finished pair waits for its cross-lane reduction
+  int e_pair = 0, e_due = 0;
+  // this group's 4 fetches: residues g_cols[k] and top-boundary rows g_rb[k]
+  const uint16_t* g_cols;
+  const uint2* g_rb;
+  auto plan_group = [&]() {   // warp-uniform
+    if (f_col == f_len) {     // the next segment starts: this group fetches its gap
+      if (f_P + 1 < passes) {
+        ++f_P;
+      } else {
+        pending = true; e_pair = f_pair; e_due = fn + 35;
+        if (nx_pair == -2) prefetch();
+        if (nx_pair >= 0) {
+          f_pair = nx_pair; f_len = nx_len; f_cols = p.cols + nx_off; f_P = 0;
+          f_pad = f_cols + (f_len - kGap);
+          nx_pair = -2;
+          if (passes == 1) prefetch();
+        } else {
+          f_pair = -1; f_len = kEndLen; f_P = -1;   // END: gap positions for ever
+        }
+      }
+      if (f_pair >= 0 && f_P == passes - 1 && passes > 1) prefetch();
+      f_col = 0;
+      ++f_seg;
+      const uint32_t d = (uint32_t)f_len | ((uint32_t)(f_P + 1) << 24);
+      if (f_seg & 1) desc1 = d; else desc0 = d;
+    }
+    if (f_col < kGap || f_pair < 0) {   // gap: pad letters (the pair's trailing pad columns)
+      g_cols = f_pad;
+      g_rb = p.rb_zero;
+    } else {
+      g_cols = f_cols + (f_col - kGap);
+      g_rb = f_P > 0 ? rb + (f_col - kGap) : p.rb_zero;
+    }
+    if (f_pair >= 0) f_col += 4;
+    fn += 4;
+  };
+  uint32_t ring_res[4], ring_h[4], ring_f[4];
+  auto fetch = [&](int k) {
+    ring_res[k] = g_cols[k];
+    const uint2 v = g_rb[k];
+    ring_h[k] = v.x; ring_f[k] = v.y;
+  };
+
+  // ---- per-lane state
+  uint32_t hrA[R], hrB[PP ? R : 1], e[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) { hrA[r] = nrho; e[r] = nrho; }
+  if constexpr (PP) {
+#pragma unroll
+    for (int r = 0; r < R; ++r) hrB[r] = nrho;
+  }
+  uint32_t hrdiag0 = nrho;
+  uint32_t y_hr = 0, y_f = 0, y_res = c.padpair;
+  uint32_t best = 0, bdone = 0;
+  int my_pos = -lane, my_len = 0, my_P = -1, my_seg = -1;   // lane l reaches segment 0 at step l
+  const uint8_t* prow = pbase;
+  bool store_rb = false;      // lane 31 in a strip whose bottom row feeds the next strip
+
+  plan_group();
+#pragma unroll
+  for (int k = 0; k < 4; ++k) fetch(k);
+
+  auto step = [&](auto kc, uint32_t* hin, uint32_t* hout) {
+    constexpr int K = decltype(kc)::value;
+    uint32_t x_hr = __shfl_up_sync(SWB_FULL, y_hr, 1);
+    uint32_t x_f = __shfl_up_sync(SWB_FULL, y_f, 1);
+    uint32_t x_res = __shfl_up_sync(SWB_FULL, y_res, 1);
+    if (lane == 0) { x_hr = ring_h[K]; x_f = ring_f[K]; x_res = ring_res[K]; }
+    uint32_t wlo[R / 4], whi[R / 4];
+    load_prof<R, CB, 32 * CB>(wlo, prow + (x_res & 0xff) * ls);
+    load_prof<R, CB, 32 * CB>(whi, prow + (x_res >> 8) * ls);
+    fetch(K);
+    uint32_t hup = x_hr, fs = x_f, hprev = 0;
+    uint32_t hrdiag = hrdiag0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {   // the cell update of run_pass
+      e[r] = L::gap(e[r], nsig, hin[r]);
+      const uint32_t u = L::hcell(hrdiag, subst_row<L, R>(wlo, whi, r), e[r]);
+      fs = L::gap(fs, nsig, hup);
+      const uint32_t h = L::gap(fs, nrho, u);
+      hrdiag = hin[r];
+      hout[r] = L::add(h, nrho);
+      hup = h;
+      if (r & 1) best = L::max3(best, hprev, h); else hprev = h;
+    }
+    hrdiag0 = L::add(x_hr, nrho);
+    y_hr = hup; y_f = fs; y_res = x_res;
+    if (store_rb) {
+      const int pos = my_pos + K;
+      if (pos >= kGap && pos < my_len) rb[pos - kGap] = make_uint2(hup, fs);
+    }
+  };
+
+  for (int S = 0;; S += 4) {
+    // switch segments: a lane whose position entered the next segment's gap
+    if (my_pos >= my_len) {
+      if (my_pos > my_len) { y_hr = 0u; y_f = 0u; }   // last step was a stale gap cell
+      ++my_seg;
+      const uint32_t d = (my_seg & 1) ? desc1 : desc0;
+      if (my_P == passes - 1) { bdone = best; best = 0; }
+      my_pos -= my_len;
+      my_len = (int)(d & (uint32_t)kEndLen);
+      my_P = (int)(d >> 24) - 1;
+      store_rb = lane == 31 && my_P >= 0 && my_P < passes - 1;
+      prow = pbase + max(my_P, 0) * kStripBytes;
+#pragma unroll
+      for (int r = 0; r < R; ++r) { hrA[r] = nrho; e[r] = nrho; }
+      hrdiag0 = nrho;
+    }
+    __syncwarp();
+    if (pending && S >= e_due) {   // every lane has parked the finished pair's maximum
+      uint32_t b = bdone;
+#pragma unroll
+      for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
+      if (lane == 0) emit<L>(p, b, e_pair, 0);
+      pending = false;
+    }
+    if (f_pair < 0 && !pending) break;
+    plan_group();   // the 4 fetches issued during this group (consumed in the next one)
+    if constexpr (PP) {
+      step(std::integral_constant<int, 0>{}, hrA, hrB);
+      step(std::integral_constant<int, 1>{}, hrB, hrA);
+      step(std::integral_constant<int, 2>{}, hrA, hrB);
+      step(std::integral_constant<int, 3>{}, hrB, hrA);
+    } else {
+      step(std::integral_constant<int, 0>{}, hrA, hrA);
+      step(std::integral_constant<int, 1>{}, hrA, hrA);
+      step(std::integral_constant<int, 2>{}, hrA, hrA);
+      step(std::integral_constant<int, 3>{}, hrA, hrA);
+    }
+    my_pos += 4;
+  }
+}
+
 template <class L, int G, int Rs, int Rl, int NT, bool PP>
 __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
   constexpr int kWarps = NT / 32;
@@ -435,6 +637,14 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
   }
 
   // ---- phase 2: GROUP (inter-task) items — short sequences, G lanes per pair
+  if constexpr (G == 32) {
+    if (p.item_list == nullptr && p.group_stream) {
+      constexpr int CBs = chunk_bytes<Rs>();
+      group_stream<L, Rs, PP>(p, c, smem + p.lg.off + lane * CBs,
+                              p.rb_group + (int64_t)(blockIdx.x * kWarps + warp) * p.rb_group_cols);
+      return;
+    }
+  }
   if (p.item_list == nullptr) {
     constexpr int GPW = 32 / G;
     const int gi = lane / G, gl = lane & (G - 1);

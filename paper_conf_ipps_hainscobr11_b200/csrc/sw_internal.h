@@ -66,6 +66,8 @@ struct SearchParams {
   // row buffers (strip bottom rows, §III "the bottom row of a strip must
   // be saved for the next pass"), uint2 = (H - rho, F) per column
   uint2* rb_group; int64_t rb_group_cols;   // per group slot (>= max n' + kPadCols)
+  int group_stream;          // G = 32: continuous stream over strips and pairs (group_stream)
+  const uint2* rb_zero;      // 4 neutral row-buffer entries (H = 0, F + rho = 0)
   uint2* rb_team;  int64_t rb_team_cols;    // per (team slot, pass mod (team_warps+1))
 };
 
