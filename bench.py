@@ -350,11 +350,15 @@ def bench_ours(args, rank, world, local_rank):
                       "CUDA-event durations, launches serialised on one stream"}
     if peaks and achieved:
         f_mhz = clk.get("sm_mhz") or peaks.get("sm_mhz_during") or 1965.0
-        per_clk = peaks["cells_per_clk_per_gpu"]
+        der = peaks["derived"]
+        per_clk = der["cells_per_clk_per_gpu"]
         peak = per_clk * f_mhz * 1e6 / 1e9
+        mix = peaks["measured_mix_cells_per_clk_per_gpu"] * f_mhz * 1e6 / 1e9
         roof.update({"peak": round(peak, 1), "frac": round(achieved / peak, 4),
-                     "peak_basis": f"measured s16x2 cell-mix issue rate {per_clk:.1f} cells/clk/GPU "
-                                   f"(MEASURED_INT_PEAKS.json) x SM clock {f_mhz:.0f} MHz during the run"})
+                     "peak_basis": f"derived ALU-pipe bound: {der['alu_pipe_warp_instr_per_clk_per_sm']} warp-instr/clk/SM "
+                                   f"(measured, = guide rt_SMSP 2) x 64 cells / {der['alu_ops_per_cell_pair']} ALU ops per "
+                                   f"cell pair = {per_clk:.1f} cells/clk/GPU x SM clock {f_mhz:.0f} MHz during the run",
+                     "measured_mix_peak": round(mix, 1), "frac_of_measured_mix": round(achieved / mix, 4)})
     prof_path = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(prof_path):
         try:

@@ -1,95 +1,144 @@
 // Integer / DPX pipe throughput microbenchmark for sm_100a (B200).
-// Defines the roofline denominator for the Smith-Waterman cell update
-// (SURVEY.md §8(d)): measured warp-instructions / clock / SM for each
-// instruction class the SW inner loop issues, plus the actual 6.5-op
-// s16x2 cell mix used by the kernels.  Output: one JSON line.
+// Defines the roofline denominator for the Smith-Waterman cell update (SURVEY.md §8(d),
+// DESIGN.md §5): measured warp-instructions / clock / SM for each instruction class the SW
+// inner loop issues, pairs of classes (which ones share a pipe), and the engine's exact s16x2
+// cell mix.  Output: one JSON line (MEASURED_INT_PEAKS.json).
 //
-//   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o int_peaks tools/int_peaks.cu -lnvidia-ml
+//   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o tools/int_peaks tools/int_peaks.cu
+//
+// Timing: every block records (smid, clock64 at start, clock64 at end) around its loop, with a
+// __syncthreads on both sides so the window covers all of its warps.  The rate of an SM is
+// (warp-instructions executed by all blocks on that SM) / (max end - min start over those
+// blocks): the SM-cycle window in which its warps actually ran, whatever the co-residency.
+// (The first version of this tool divided each block's own window into an assumed
+// co-resident warp count, which over-stated every rate by ~1.33x when the two blocks of an SM
+// did not overlap completely: ncu measured 92 % ALU-pipe activity for the cell mix at a rate
+// 0.75x of what that version reported.)  Each op's operands come from other chains, and the
+// ops are asm volatile, so nothing folds.
 #include <cstdio>
 #include <cstdint>
+#include <vector>
 #include <algorithm>
 #include <cuda_runtime.h>
 
 #define CHAINS 8
-#define ITERS 4096
+#define ITERS 2048
+
+struct Rec { long long t0, t1; unsigned long long g0, g1; unsigned smid; unsigned pad; };
 
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
   return t;
 }
-
-template <int OP>
-__device__ __forceinline__ uint32_t op(uint32_t a, uint32_t b, uint32_t c) {
-  if constexpr (OP == 0) return __viaddmax_s16x2(a, b, c);          // VIADDMNMX.S16x2
-  if constexpr (OP == 1) return __vimax3_s16x2_relu(a, b, c);       // VIMNMX3.S16x2.RELU
-  if constexpr (OP == 2) return __vmaxs2(a, c);                     // VIMNMX.S16x2
-  if constexpr (OP == 3) return __vadd2(a, b);                      // VIADD.16x2
-  if constexpr (OP == 4) return __byte_perm(a, c, 0xC480);          // PRMT
-  if constexpr (OP == 5) return a + b + c;                          // IADD3
-  if constexpr (OP == 6) return (uint32_t)max((int)a, (int)c);      // IMNMX
-  if constexpr (OP == 7) return __viaddmax_s16x2_relu(a, b, c);     // VIADDMNMX.S16x2.RELU
-  if constexpr (OP == 8) return (uint32_t)__viaddmax_s32((int)a, (int)b, (int)c);  // VIADDMNMX (s32)
-  return a;
+__device__ __forceinline__ unsigned smid() {
+  unsigned s;
+  asm volatile("mov.u32 %0, %smid;" : "=r"(s));
+  return s;
 }
 
+// one instruction of class OP (asm volatile: never folded, never hoisted)
 template <int OP>
-__global__ void __launch_bounds__(512) k_peak(uint32_t* out, uint32_t seed, long long* cyc) {
+__device__ __forceinline__ uint32_t op(uint32_t a, uint32_t b, uint32_t c) {
+  uint32_t d;
+  if constexpr (OP == 2) asm volatile("prmt.b32 %0, %1, %2, 0xC480;" : "=r"(d) : "r"(a), "r"(c));
+  if constexpr (OP == 3) asm volatile("add.s32 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(c));
+  if constexpr (OP == 4) asm volatile("lop3.b32 %0, %1, %2, %3, 0x96;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+  if constexpr (OP == 5) asm volatile("max.s32 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(c));
+  if constexpr (OP == 6) asm volatile("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+  return d;
+}
+// DPX classes through the intrinsics (ptxas emits one SASS op each); volatile via a barrier
+// on the result so the compiler keeps every one.
+template <int OP>
+__device__ __forceinline__ uint32_t dpx(uint32_t a, uint32_t b, uint32_t c) {
+  uint32_t d;
+  if constexpr (OP == 10) d = __viaddmax_s16x2(a, b, c);          // VIADDMNMX.S16x2
+  if constexpr (OP == 11) d = __viaddmax_s16x2_relu(a, b, c);     // VIADDMNMX.S16x2.RELU
+  if constexpr (OP == 12) d = __vimax3_s16x2(a, b, c);            // VIMNMX3.S16x2
+  if constexpr (OP == 13) d = __vmaxs2(a, c);                     // VIMNMX.S16x2
+  if constexpr (OP == 14) d = __vadd2(a, b);                      // VIADD.16x2 (HADD2-class?)
+  if constexpr (OP == 15) d = (uint32_t)__viaddmax_s32((int)a, (int)b, (int)c);
+  if constexpr (OP < 10) d = op<OP>(a, b, c);
+  asm volatile("" : "+r"(d));
+  return d;
+}
+
+// OPA on every chain; if OPB >= 0, chains alternate OPA / OPB (pipe-sharing test)
+template <int OPA, int OPB>
+__global__ void __launch_bounds__(512) k_peak(uint32_t* out, uint32_t seed, Rec* rec) {
   uint32_t v[CHAINS];
 #pragma unroll
-  for (int k = 0; k < CHAINS; ++k) v[k] = seed * (threadIdx.x + 1) + k;
-  uint32_t b = seed ^ 0x00030003u, c = seed ^ 0x00070007u;
+  for (int k = 0; k < CHAINS; ++k) v[k] = seed * (threadIdx.x + 1) + k * 0x00010003u;
+  const uint32_t b = seed ^ 0xFFFEFFFEu;
+  __syncthreads();
   long long t0 = clock64();
   unsigned long long g0 = gtimer();
   for (int it = 0; it < ITERS; ++it) {
 #pragma unroll
-    for (int k = 0; k < CHAINS; ++k) v[k] = op<OP>(v[k], b, c ^ k);
+    for (int k = 0; k < CHAINS; ++k) {
+      const uint32_t c = v[(k + 1) % CHAINS];
+      if (OPB < 0 || (k & 1) == 0) v[k] = dpx<OPA>(v[k], b, c);
+      else v[k] = dpx<(OPB < 0 ? OPA : OPB)>(v[k], b, c);
+    }
   }
+  __syncthreads();
   long long t1 = clock64();
   unsigned long long g1 = gtimer();
   uint32_t acc = 0;
 #pragma unroll
   for (int k = 0; k < CHAINS; ++k) acc ^= v[k];
   if (acc == 0x12345678u) out[blockIdx.x * blockDim.x + threadIdx.x] = acc;
-  if (threadIdx.x == 0) { cyc[2 * blockIdx.x] = t1 - t0; cyc[2 * blockIdx.x + 1] = (long long)(g1 - g0); }
+  if (threadIdx.x == 0) rec[blockIdx.x] = Rec{t0, t1, g0, g1, smid(), 0};
 }
 
-// The s16x2 Smith-Waterman cell update exactly as sw_engine.cuh issues it (per row: PRMT +
-// VIADDMNMX x2 + VIMNMX + VIADDMNMX.RELU + VIADD + 0.5 VIMNMX3), profile words varying per
-// column, no memory traffic: the ALU speed of light of the engine's arithmetic.
+// The s16x2 Smith-Waterman cell update exactly as sw_engine.cuh's run_pass issues it, per row:
+//   e  = VIADDMNMX(e, -sigma, hr_left)
+//   u  = VIADDMNMX.RELU(hr_diag, w + rho, e)
+//   fs = VIADDMNMX(fs, -sigma, h_up)
+//   h  = VIADDMNMX(fs, -rho, u)
+//   hr = VIADD.16x2(h, -rho)
+//   w  = PRMT(profile_lo, profile_hi)          (sign-extend two int8 scores)
+//   best = VIMNMX3(best, h, h') every two rows
+// = 6.5 ALU-class instructions per two cells; the profile words come from shared memory (LDS.128,
+// R/16 x 2 per column as in the engine) at a letter that changes every column.
 template <uint32_t SEL>
 __device__ __forceinline__ uint32_t prmt_imm(uint32_t a, uint32_t b) {
   uint32_t d;
   asm("prmt.b32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "n"(SEL));
   return d;
 }
-constexpr int CM_R = 16;
-__global__ void __launch_bounds__(512) k_cellmix(uint32_t* out, uint32_t seed, long long* cyc) {
+constexpr int CM_R = 32;
+constexpr int CM_COLS = 256;
+__global__ void __launch_bounds__(512) k_cellmix(uint32_t* out, uint32_t seed, Rec* rec) {
   constexpr int R = CM_R;
   uint32_t hr[R], e[R];
-#pragma unroll
-  for (int r = 0; r < R; ++r) { hr[r] = 0xFFF6FFF6u; e[r] = 0xFFF6FFF6u; }
-  uint32_t best = 0, hrup0 = 0xFFF6FFF6u, f0 = 0xFFF6FFF6u, hrdiag0 = 0xFFF6FFF6u;
   const uint32_t nsig = 0xFFFEFFFEu, nrho = 0xFFF6FFF6u;
-  // profile rows in shared memory, read with LDS.128 exactly like the engine (25 letters)
-  __shared__ __align__(16) uint32_t sprof[25 * R];
-  for (int i = threadIdx.x; i < 25 * R; i += blockDim.x) sprof[i] = (seed + i) * 0x01010101u;
+#pragma unroll
+  for (int r = 0; r < R; ++r) { hr[r] = nrho; e[r] = nrho; }
+  uint32_t best = 0, hup0 = 0, fs0 = 0, hrdiag0 = nrho;
+  // profile: 16 letters x R rows of int8, per-lane copy so the LDS.128 are conflict-free
+  __shared__ __align__(16) uint8_t sprof[16 * R * 32];
+  for (int i = threadIdx.x; i < 16 * R * 32; i += blockDim.x) sprof[i] = (uint8_t)((seed + i * 37u) % 23u);
+  // the residue stream (two letters per column), in shared memory like a staged DB tile
+  __shared__ uint8_t sres[CM_COLS];
+  for (int i = threadIdx.x; i < CM_COLS; i += blockDim.x) sres[i] = (uint8_t)((i * 0x9Du + seed) & 0xffu);
   __syncthreads();
-  uint32_t res = threadIdx.x * 7u + seed;
+  const int lane = threadIdx.x & 31;
   long long t0 = clock64();
   unsigned long long g0 = gtimer();
-  for (int it = 0; it < ITERS / 8; ++it) {
+  for (int col = 0; col < ITERS / 4; ++col) {
+    const uint32_t res = sres[col & (CM_COLS - 1)];
+    const uint4* plo = reinterpret_cast<const uint4*>(sprof + ((res & 15) * R * 32)) + lane;
+    const uint4* phi = reinterpret_cast<const uint4*>(sprof + ((res >> 4) * R * 32)) + lane;
     uint32_t wlo[R / 4], whi[R / 4];
-    const uint4* plo = reinterpret_cast<const uint4*>(sprof + (res & 15) * R);
-    const uint4* phi = reinterpret_cast<const uint4*>(sprof + ((res >> 4) & 15) * R);
 #pragma unroll
     for (int k = 0; k < R / 16; ++k) {
-      const uint4 a = plo[k], b = phi[k];
+      const uint4 a = plo[k * 32], bb = phi[k * 32];
       wlo[4 * k] = a.x; wlo[4 * k + 1] = a.y; wlo[4 * k + 2] = a.z; wlo[4 * k + 3] = a.w;
-      whi[4 * k] = b.x; whi[4 * k + 1] = b.y; whi[4 * k + 2] = b.z; whi[4 * k + 3] = b.w;
+      whi[4 * k] = bb.x; whi[4 * k + 1] = bb.y; whi[4 * k + 2] = bb.z; whi[4 * k + 3] = bb.w;
     }
-    res = res * 0x9E37u + 0x79B9u;
-    uint32_t hrup = hrup0, f = f0, hrdiag = hrdiag0, hprev = 0;
+    uint32_t hup = hup0, fs = fs0, hrdiag = hrdiag0, hprev = 0;
 #pragma unroll
     for (int r = 0; r < R; ++r) {
       uint32_t w;
@@ -100,91 +149,109 @@ __global__ void __launch_bounds__(512) k_cellmix(uint32_t* out, uint32_t seed, l
         default: w = prmt_imm<0xF7B3u>(wlo[r >> 2], whi[r >> 2]); break;
       }
       e[r] = __viaddmax_s16x2(e[r], nsig, hr[r]);
-      f = __viaddmax_s16x2(f, nsig, hrup);
-      const uint32_t ef = __vmaxs2(e[r], f);
-      const uint32_t h = __viaddmax_s16x2_relu(hrdiag, w, ef);
+      const uint32_t u = __viaddmax_s16x2_relu(hrdiag, w, e[r]);
+      fs = __viaddmax_s16x2(fs, nsig, hup);
+      const uint32_t h = __viaddmax_s16x2(fs, nrho, u);
       hrdiag = hr[r];
       hr[r] = __vadd2(h, nrho);
-      hrup = hr[r];
+      hup = h;
       if (r & 1) best = __vimax3_s16x2(best, hprev, h); else hprev = h;
     }
-    hrdiag0 = hrup0; hrup0 = hrup ^ (uint32_t)it; f0 = f;
+    // the next column's top input: this lane's bottom row (a chain of one lane)
+    hrdiag0 = __vadd2(hup0, nrho);
+    hup0 = hup; fs0 = fs;
   }
+  __syncthreads();
   long long t1 = clock64();
   unsigned long long g1 = gtimer();
   uint32_t acc = best;
 #pragma unroll
   for (int r = 0; r < R; ++r) acc ^= hr[r] ^ e[r];
   if (acc == 0x12345678u) out[blockIdx.x * blockDim.x + threadIdx.x] = acc;
-  if (threadIdx.x == 0) { cyc[2 * blockIdx.x] = t1 - t0; cyc[2 * blockIdx.x + 1] = (long long)(g1 - g0); }
+  if (threadIdx.x == 0) rec[blockIdx.x] = Rec{t0, t1, g0, g1, smid(), 0};
 }
 
-static double g_last_rate = 0, g_last_clk = 0;
-// Rate in warp-instructions per SM clock: all blocks resident (one wave), per-block SM cycles
-// from clock64 and wall time from %globaltimer give the clock the kernel actually ran at; the
-// GPU is warmed up for ~1.5 s first so the clock has ramped (an earlier version of this tool
-// measured a cold GPU and under-estimated the clock).
+static double g_rate = 0, g_clk = 0;
+// work_per_thread: instructions (or cells) per thread of the timed loop
 template <typename K>
-static void run(const char* name, K kern, double instr_per_thread, int blocks, int threads, uint32_t* d_out,
-                long long* d_cyc, int first) {
+static void run(const char* name, K kern, double work_per_thread, int threads, uint32_t* d_out, Rec* d_rec,
+                bool first) {
+  int nsm = 0; cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, 0);
+  int occ = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, threads, 0);
+  occ = std::max(1, std::min(occ, 4));
+  const int blocks = nsm * occ;                       // one resident wave
   cudaEvent_t a, b;
   cudaEventCreate(&a); cudaEventCreate(&b);
   cudaEventRecord(a);
-  int warm = 0;
-  for (;;) {
-    kern<<<blocks, threads>>>(d_out, 1u + warm, d_cyc);
-    ++warm;
+  for (int warm = 0;; ++warm) {                       // ~1 s warm-up so the clock has ramped
+    kern<<<blocks, threads>>>(d_out, 1u + warm, d_rec);
     cudaEventRecord(b);
     cudaEventSynchronize(b);
     float ms = 0; cudaEventElapsedTime(&ms, a, b);
-    if (ms > 1500.f || warm > 20000) break;
+    if (ms > 1000.f || warm > 20000) break;
   }
-  const int reps = 20;
+  const int reps = 10;
+  std::vector<Rec> h(blocks);
   double sum_rate = 0, sum_clk = 0;
   for (int i = 0; i < reps; ++i) {
-    kern<<<blocks, threads>>>(d_out, 7u + i, d_cyc);
-    static long long h_cyc[2 * 8192];
-    cudaMemcpy(h_cyc, d_cyc, sizeof(long long) * 2 * blocks, cudaMemcpyDeviceToHost);
-    double cyc = 0, ns = 0;
-    for (int k = 0; k < blocks; ++k) { cyc += (double)h_cyc[2 * k]; ns += (double)h_cyc[2 * k + 1]; }
-    const double clk_ghz = cyc / ns;                 // SM cycles per ns inside the timed loop
-    int nsm = 0; cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, 0);
-    const double warps_per_sm = (double)blocks * threads / 32.0 / nsm;
-    sum_rate += warps_per_sm * instr_per_thread / (cyc / blocks);
-    sum_clk += clk_ghz;
+    kern<<<blocks, threads>>>(d_out, 7u + i, d_rec);
+    cudaMemcpy(h.data(), d_rec, sizeof(Rec) * blocks, cudaMemcpyDeviceToHost);
+    std::vector<long long> lo(nsm, INT64_MAX), hi(nsm, INT64_MIN);
+    std::vector<unsigned long long> glo(nsm, UINT64_MAX), ghi(nsm, 0);
+    std::vector<int> nb(nsm, 0);
+    for (auto& r : h) {
+      if (r.smid >= (unsigned)nsm) continue;
+      lo[r.smid] = std::min(lo[r.smid], r.t0); hi[r.smid] = std::max(hi[r.smid], r.t1);
+      glo[r.smid] = std::min(glo[r.smid], r.g0); ghi[r.smid] = std::max(ghi[r.smid], r.g1);
+      nb[r.smid]++;
+    }
+    double rate = 0, clk = 0; int used = 0;
+    for (int s = 0; s < nsm; ++s) {
+      if (!nb[s]) continue;
+      const double cyc = (double)(hi[s] - lo[s]);
+      rate += nb[s] * (threads / 32.0) * work_per_thread / cyc;
+      clk += cyc / (double)(ghi[s] - glo[s]);
+      ++used;
+    }
+    sum_rate += rate / used; sum_clk += clk / used;
   }
-  const double rate = sum_rate / reps, clk = sum_clk / reps;
-  g_last_rate = rate; g_last_clk = clk;
-  printf("%s\"%s\": {\"warp_instr_per_clk_per_sm\": %.3f, \"sm_clock_ghz\": %.3f}", first ? "" : ", ", name, rate, clk);
+  g_rate = sum_rate / reps; g_clk = sum_clk / reps;
+  printf("%s\"%s\": {\"warp_instr_per_clk_per_sm\": %.3f, \"sm_clock_ghz\": %.3f, \"blocks_per_sm\": %d}",
+         first ? "" : ", ", name, g_rate, g_clk, occ);
+  fflush(stdout);
 }
 
 int main() {
   int nsm = 0; cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, 0);
   const int threads = 512;
-  int occ = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_cellmix, threads, 0);
-  const int blocks = nsm * std::max(1, std::min(occ, 2));   // one resident wave
-  uint32_t* d_out; long long* d_cyc;
-  cudaMalloc(&d_out, sizeof(uint32_t) * blocks * threads);
-  cudaMalloc(&d_cyc, sizeof(long long) * 2 * blocks);
+  uint32_t* d_out; Rec* d_rec;
+  cudaMalloc(&d_out, sizeof(uint32_t) * nsm * 4 * threads);
+  cudaMalloc(&d_rec, sizeof(Rec) * nsm * 4);
   const double ipt = (double)CHAINS * ITERS;
   printf("{\"sms\": %d, ", nsm);
-  run("VIADDMNMX.S16x2", k_peak<0>, ipt, blocks, threads, d_out, d_cyc, 1);
-  run("VIMNMX3.S16x2.RELU", k_peak<1>, ipt, blocks, threads, d_out, d_cyc, 0);
-  run("VIMNMX.S16x2", k_peak<2>, ipt, blocks, threads, d_out, d_cyc, 0);
-  run("VIADD.16x2", k_peak<3>, ipt, blocks, threads, d_out, d_cyc, 0);
-  run("PRMT", k_peak<4>, ipt, blocks, threads, d_out, d_cyc, 0);
-  run("IADD3", k_peak<5>, ipt, blocks, threads, d_out, d_cyc, 0);
-  run("IMNMX", k_peak<6>, ipt, blocks, threads, d_out, d_cyc, 0);
-  run("VIADDMNMX.S16x2.RELU", k_peak<7>, ipt, blocks, threads, d_out, d_cyc, 0);
-  run("VIADDMNMX.S32", k_peak<8>, ipt, blocks, threads, d_out, d_cyc, 0);
-  // cell mix, counted in CELLS: per iteration R rows x 2 cells (two sequences per s16x2 lane)
-  run("cellmix_cells", k_cellmix, (ITERS / 8) * CM_R * 2.0, blocks, threads, d_out, d_cyc, 0);
-  // g_last_rate is "warp-cells" per clk per SM -> x32 lanes x SMs = cells per clk per GPU
-  printf(", \"cells_per_clk_per_gpu\": %.2f, \"sm_mhz_during\": %.0f, \"what\": \"cells_per_clk_per_gpu = measured rate "
-         "of the engine's per-cell instruction mix (PRMT + 5 DPX + 0.5 VIMNMX3 per 2 cells, profile from smem), no "
-         "boundary traffic; the DPX ops issue at the rate measured for VIADDMNMX.S16x2 above\"}\n",
-         g_last_rate * 32.0 * nsm, g_last_clk * 1e3);
+  run("VIADDMNMX.S16x2", k_peak<10, -1>, ipt, threads, d_out, d_rec, true);
+  run("VIADDMNMX.S16x2.RELU", k_peak<11, -1>, ipt, threads, d_out, d_rec, false);
+  run("VIMNMX3.S16x2", k_peak<12, -1>, ipt, threads, d_out, d_rec, false);
+  run("VIMNMX.S16x2", k_peak<13, -1>, ipt, threads, d_out, d_rec, false);
+  run("VIADD.16x2", k_peak<14, -1>, ipt, threads, d_out, d_rec, false);
+  run("VIADDMNMX.S32", k_peak<15, -1>, ipt, threads, d_out, d_rec, false);
+  run("PRMT", k_peak<2, -1>, ipt, threads, d_out, d_rec, false);
+  run("IADD3", k_peak<3, -1>, ipt, threads, d_out, d_rec, false);
+  run("LOP3", k_peak<4, -1>, ipt, threads, d_out, d_rec, false);
+  run("IMNMX", k_peak<5, -1>, ipt, threads, d_out, d_rec, false);
+  run("IMAD", k_peak<6, -1>, ipt, threads, d_out, d_rec, false);
+  // pipe sharing: the pair's combined rate is ~1 pipe's rate if both go to the same pipe
+  run("VIADDMNMX+PRMT", k_peak<10, 2>, ipt, threads, d_out, d_rec, false);
+  run("VIADDMNMX+VIADD.16x2", k_peak<10, 14>, ipt, threads, d_out, d_rec, false);
+  run("VIADDMNMX+IMAD", k_peak<10, 6>, ipt, threads, d_out, d_rec, false);
+  run("VIADDMNMX+IADD3", k_peak<10, 3>, ipt, threads, d_out, d_rec, false);
+  // the cell mix, counted in CELLS: per column R rows x 2 cells (two sequences per s16x2 lane)
+  run("cellmix_cells", k_cellmix, (ITERS / 4) * CM_R * 2.0, threads, d_out, d_rec, false);
+  printf(", \"cells_per_clk_per_gpu\": %.2f, \"sm_mhz_during\": %.0f, \"what\": \"rates = warp-instructions (cellmix: "
+         "warp-cells) per SM clock over the per-SM window in which the blocks ran; cells_per_clk_per_gpu = 32 lanes x "
+         "SMs x the cell-mix rate (PRMT + 5 DPX + 0.5 VIMNMX3 per 2 cells, profile from smem via LDS.128)\"}\n",
+         g_rate * 32.0 * nsm, g_clk * 1e3);
   cudaError_t err = cudaGetLastError();
   if (err != cudaSuccess) { fprintf(stderr, "CUDA error %s\n", cudaGetErrorString(err)); return 1; }
   return 0;
