@@ -156,6 +156,10 @@ int grow(sw_handle h, T** p, size_t* cap, size_t bytes, const char* what, cudaSt
   if (bytes == 0) return SW_OK;
   cudaError_t e = cudaMalloc(reinterpret_cast<void**>(p), bytes);
   if (e != cudaSuccess) return cuda_fail(h, e, what);
+  // zero-filled: the row buffers' leading slot of every strip buffer must read as the neutral
+  // entry (H, F + rho) = (0, 0) (run_pass); it is only ever rewritten with neutral values
+  e = busy ? cudaMemsetAsync(*p, 0, bytes, busy) : cudaMemset(*p, 0, bytes);
+  if (e != cudaSuccess) return cuda_fail(h, e, what);
   *cap = bytes;
   return SW_OK;
 }
@@ -175,9 +179,10 @@ ProfLayout make_layout(int off, int G, int R, int m, int A1, int nrep) {
   L.off = off;
   L.G = G;
   L.R = R;
-  L.cb = (R % 8 == 0) ? 8 : 4;
+  L.cb = (R >= 12) ? 16 : (R % 8 == 0) ? 8 : 4;   // == chunk_bytes<R>() (sw_engine.cuh)
+  L.nch = (R + L.cb - 1) / L.cb;
   L.strips = (m + G * R - 1) / (G * R);
-  L.ls = (int)round_up((int64_t)L.strips * G * R, 128);
+  L.ls = (int)round_up((int64_t)L.strips * L.nch * G * L.cb, 128);
   L.nrep = nrep;
   L.rs = (int)round_up((int64_t)A1 * L.ls, 128) + (nrep > 1 ? (L.cb * G) % 128 : 0);
   L.bytes = (int)round_up((int64_t)(nrep - 1) * L.rs + (int64_t)A1 * L.ls, 128);
@@ -425,8 +430,9 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   rc = grow(h, &s.d_ovf_list, &ovf_cap, ovf_bytes, "alloc overflow list", s.stream);
   if (rc) return rc;
   s.ovf_cap = (int64_t)(ovf_cap / sizeof(int32_t));
-  const int64_t max_cols_all = h->db->n_pairs ? h->db->h_pair_ncols[0] + kPadCols : 0;
-  const int64_t max_cols_short = (n_long < h->db->n_pairs) ? h->db->h_pair_ncols[n_long] + kPadCols : 0;
+  // row-buffer slots: the pair's columns (+ pad tail) plus one leading neutral entry
+  const int64_t max_cols_all = h->db->n_pairs ? h->db->h_pair_ncols[0] + kPadCols + 1 : 0;
+  const int64_t max_cols_short = (n_long < h->db->n_pairs) ? h->db->h_pair_ncols[n_long] + kPadCols + 1 : 0;
   const int G = pl.cfg.G;
   size_t rbg = 0;
   if (pl.short_passes > 1 && max_cols_short > 0)
@@ -460,7 +466,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
     rc = grow(h, &s.d_qpair, &s.qpair_cap, (size_t)(qcols + kPadCols) * sizeof(uint16_t), "alloc query stream",
               s.stream);
     if (rc) return rc;
-    rc = grow(h, &s.d_rb_t, &s.rb_t_cap, (size_t)t_grid * 2 * t_warps * (qcols + kPadCols) * sizeof(uint2),
+    rc = grow(h, &s.d_rb_t, &s.rb_t_cap, (size_t)t_grid * 2 * t_warps * (qcols + kPadCols + 1) * sizeof(uint2),
               "alloc long-sequence row buffers", s.stream);
     if (rc) return rc;
   }
@@ -545,7 +551,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
     t.big_strips = 16;
     if (const char* f = getenv("SW_T_BIG")) t.big_strips = std::max(1, atoi(f));
     t.rb = s.d_rb_t;
-    t.rb_cols = qcols + kPadCols;
+    t.rb_cols = qcols + kPadCols + 1;
     SW_CUDA(h, launch_tmode(t, t_grid, t_smem, s.aux));
     SW_CUDA(h, cudaEventRecord(s.join, s.aux));
   }
@@ -611,7 +617,7 @@ int build_db(sw_handle h, DbState& db, const uint8_t* residues, const int64_t* o
   db.sorted_len.resize((size_t)num_seqs);
   for (int64_t k = 0; k < num_seqs; ++k) db.sorted_len[k] = len[perm[k]];
   const int n_pairs = (int)((num_seqs + 1) / 2);
-  db.h_pair_off.assign((size_t)n_pairs + 1, 0);
+  db.h_pair_off.assign((size_t)n_pairs + 1, kLeadCols);
   db.h_pair_ncols.assign((size_t)n_pairs, 0);
   for (int p = 0; p < n_pairs; ++p) {
     const int64_t lo = db.sorted_len[2 * p];
@@ -645,6 +651,7 @@ int build_db(sw_handle h, DbState& db, const uint8_t* residues, const int64_t* o
     cols = cols_vec.data();
   }
   const uint16_t pad = (uint16_t)h->A;
+  for (int j = 0; j < kLeadCols; ++j) cols[j] = (uint16_t)(pad | (pad << 8));
   auto pack = [&](int p0, int p1) {
     for (int p = p0; p < p1; ++p) {
       uint16_t* dst = cols + db.h_pair_off[p];

@@ -151,11 +151,28 @@ __device__ __forceinline__ void team_bar(int team, int W) {
 
 // R rows of one letter for one lane -> R/4 words (4 query rows per word, §III-B
 // "stores the similarity scores of four symbols in a single variable").  The lane's rows are
-// R/CB chunks of CB bytes, STRIDE bytes apart (ProfLayout).
+// chunks of CB bytes, STRIDE bytes apart (ProfLayout); with CB = 16 the last chunk may be
+// partial (R % 16 rows), read with the narrowest load that covers it.
 template <int R, int CB, int STRIDE>
 __device__ __forceinline__ void load_prof(uint32_t (&w)[R / 4], const uint8_t* p) {
-  static_assert(R % CB == 0, "R must be a multiple of the chunk size");
-  if constexpr (CB == 8) {
+  if constexpr (CB == 16) {
+#pragma unroll
+    for (int k = 0; k < R / 16; ++k) {
+      const uint4 v = *reinterpret_cast<const uint4*>(p + k * STRIDE);
+      w[4 * k + 0] = v.x; w[4 * k + 1] = v.y; w[4 * k + 2] = v.z; w[4 * k + 3] = v.w;
+    }
+    constexpr int k = R / 16, rem = (R % 16) / 4;
+    if constexpr (rem == 3) {
+      const uint4 v = *reinterpret_cast<const uint4*>(p + k * STRIDE);
+      w[4 * k + 0] = v.x; w[4 * k + 1] = v.y; w[4 * k + 2] = v.z;
+    } else if constexpr (rem == 2) {
+      const uint2 v = *reinterpret_cast<const uint2*>(p + k * STRIDE);
+      w[4 * k + 0] = v.x; w[4 * k + 1] = v.y;
+    } else if constexpr (rem == 1) {
+      w[4 * k] = *reinterpret_cast<const uint32_t*>(p + k * STRIDE);
+    }
+  } else if constexpr (CB == 8) {
+    static_assert(R % 8 == 0, "R must be a multiple of the chunk size");
 #pragma unroll
     for (int k = 0; k < R / 8; ++k) {
       const uint2 v = *reinterpret_cast<const uint2*>(p + k * STRIDE);
@@ -167,8 +184,12 @@ __device__ __forceinline__ void load_prof(uint32_t (&w)[R / 4], const uint8_t* p
   }
 }
 
+// Profile chunk size for R rows per lane: 16-byte chunks (LDS.128, the last one partial when
+// R % 16 != 0) from 12 rows up, else 8 or 4.  Must match make_layout (sw_api.cu).
 template <int R>
-__host__ __device__ constexpr int chunk_bytes() { return (R % 8 == 0) ? 8 : 4; }
+__host__ __device__ constexpr int chunk_bytes() { return (R >= 12) ? 16 : (R % 8 == 0) ? 8 : 4; }
+template <int R>
+__host__ __device__ constexpr int chunks_per_lane() { return (R + chunk_bytes<R>() - 1) / chunk_bytes<R>(); }
 
 // substitution value (w + rho) of row r of the lane's window, packed per Lane
 template <class L, int R>
@@ -192,13 +213,49 @@ struct ChainConst {
   uint32_t padpair;       // residue pair of two pad letters
 };
 
+// The cell update (one row r of one column j, both sequences of the pair), in the
+// "look-ahead" form used by every mode: besides E, each row keeps u = max(H[r-1][j] + w(q_r,
+// d_{j+1}), E[r][j+1], 0) for the NEXT column, formed as soon as its inputs exist (the row
+// above's H at this column and this row's new E).  Then every per-row register (e[r], u[r]) is
+// read and rewritten by its own row only, so the unrolled step loop needs no register
+// rotation (the previous form kept H - rho of the left column per row, whose old value had to
+// survive one row longer than its new one: ~R register moves per step, or 2R registers).
+//   fs   = max(fs - sigma, h_up)          F + rho of this row      VIADDMNMX
+//   h    = max(fs - rho, u[r])            H[r][j]                  VIADDMNMX
+//   hr   = h - rho                                                 VIADD.16x2 (FMA pipe)
+//   e[r] = max(e[r] - sigma, hr)          E[r][j+1]                VIADDMNMX
+//   u[r] = max(hr_up + (w + rho), e[r], 0)  for column j+1         VIADDMNMX.RELU
+//   best = max(best, h, h') every two rows                         VIMNMX3
+// plus one PRMT per row for w + rho of column j+1 (profile words of the next column's letters).
+template <class L, int R>
+__device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&u)[R], const uint32_t (&wlo)[R / 4],
+                                          const uint32_t (&whi)[R / 4], uint32_t nrho, uint32_t nsig,
+                                          uint32_t& hup, uint32_t& fs, uint32_t& best) {
+  uint32_t hrup = L::add(hup, nrho), hprev = 0;
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    fs = L::gap(fs, nsig, hup);                                       // F + rho = max(F[i-1] + rho - sigma, H[i-1])
+    const uint32_t h = L::gap(fs, nrho, u[r]);                        // H = max(F, u)
+    const uint32_t hr = L::add(h, nrho);                              // H - rho
+    e[r] = L::gap(e[r], nsig, hr);                                    // E[j+1] = max(E - sigma, H - rho)
+    u[r] = L::hcell(hrup, subst_row<L, R>(wlo, whi, r), e[r]);        // max(H[i-1][j] + w(q_i, d_{j+1}), E[j+1], 0)
+    hrup = hr;
+    hup = h;
+    if (r & 1) best = L::max3(best, hprev, h); else hprev = h;
+  }
+}
+
 // One strip pass of a chain of GC lanes over the columns of one database pair (see the file
 // header).  Lane l owns rows [(P*GC + l)*R, +R) of the query and processes column j at step
-// j + l.  All lanes start the pass in the neutral state (H = 0 -> hr = -rho, E = -inf -> -rho
-// by reading c4); a lane still in its pipeline fill sees neutral inputs and pad letters, which
-// keep it exactly neutral, so no per-lane reset is needed inside the step loop.
-// Returns max(best, this lane's H maxima) (packed per Lane).
-template <class L, int GC, int R, bool TEAM, bool PP>
+// j + l + 1: every lane (lane 0 included) first processes one pad column j = -1 in the neutral
+// state, whose look-ahead forms u for column 0.  All lanes start the pass in the neutral state
+// (H = 0, E = -inf -> -rho by reading c4, u = 0); a lane still in its pipeline fill sees
+// neutral inputs and pad letters, which keep it exactly neutral, so no per-lane reset is
+// needed inside the step loop.  The residue stream each lane receives is one column ahead (the
+// letters of column j + 1, for the profile of u).  rb_in[-1] must be a neutral entry (0, 0)
+// (the row buffers carry one leading slot, zero-initialised and only ever rewritten with the
+// neutral fill values).  Returns max(best, this lane's H maxima) (packed per Lane).
+template <class L, int GC, int R, bool TEAM>
 __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t* prow, int ls, int hi_off,
                                              const uint16_t* __restrict__ cols, int ncols,
                                              int half, int steps, int P, int passes_total,
@@ -214,33 +271,23 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
   const bool store_out = (gl == GC - 1) && (P < passes_total - 1);
   const bool from_prev = P > 0;
 
-  // PP: the unrolled step loop ping-pongs between two register arrays (H - rho of the left
-  // column / of this column) so the allocator needs fewer copies (§III-A: keep
-  // the tile in registers); without PP one array is updated in place (fewer registers, more
-  // resident warps, some register moves on the FMA pipe).
-  uint32_t hrA[R], hrB[PP ? R : 1], e[R];
+  uint32_t e[R], u[R];
 #pragma unroll
-  for (int r = 0; r < R; ++r) { hrA[r] = nrho; e[r] = nrho; }
-  if constexpr (PP) {
-#pragma unroll
-    for (int r = 0; r < R; ++r) hrB[r] = nrho;
-  }
-  // neutral state: H = 0 on the row above / left column, E = F = -rho (<= 0, reading c4)
-  uint32_t hrdiag0 = nrho;
+  for (int r = 0; r < R; ++r) { e[r] = nrho; u[r] = 0u; }
   uint32_t y_hr = 0, y_f = 0, y_res = c.padpair;   // (H, F + rho) of this lane's bottom row
-  int col = -gl;
+  int col = -gl - 1;
 
-  // Lane 0 streams residues and the previous strip's bottom row through a 4-deep register
-  // ring: the loads for column j + 4 are issued while column j is computed, so L2 latency is
-  // hidden behind four steps of DP work.  Every pair is stored with kPadCols trailing pad
-  // columns, so the stream runs branch-free past the last column (clamped to the last pad
-  // column): the lanes then compute the DP of the sequence extended by pad letters, whose
-  // optimum is the same (a pad column only adds -128 substitutions or gaps, so truncating an
-  // alignment at the last real column never lowers its score).  The previous strip's last
-  // lane wrote columns 0 .. steps - GC; later columns reuse the last one (bounded, legitimate
-  // DP values of the extended matrix).
+  // Lane 0 streams residues (one column ahead) and the previous strip's bottom row through a
+  // 4-deep register ring: the loads for step s + 4 are issued while step s is computed, so L2
+  // latency is hidden behind four steps of DP work.  Every pair is stored with kPadCols
+  // trailing pad columns, so the stream runs branch-free past the last column (clamped to the
+  // last pad column): the lanes then compute the DP of the sequence extended by pad letters,
+  // whose optimum is the same (a pad column only adds -128 substitutions or gaps, so
+  // truncating an alignment at the last real column never lowers its score).  The previous
+  // strip's last lane wrote columns -1 .. steps - GC - 1; later columns reuse the last one
+  // (bounded, legitimate DP values of the extended matrix).
   const int cmax = ncols + kPadCols - 1;
-  const int rlast = steps - GC;
+  const int rlast = steps - GC - 1;
   uint32_t ring_res[4], ring_h[4], ring_f[4];   // top boundary: H[0][j] = 0, F[0][j] + rho <= 0
 #pragma unroll
   for (int k = 0; k < 4; ++k) { ring_res[k] = c.padpair; ring_h[k] = 0; ring_f[k] = 0; }
@@ -248,9 +295,9 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
   // Every lane of the chain runs the fetch (same addresses as its lane 0: broadcast loads, no
   // extra traffic) so the warp never diverges; only lane 0 consumes the values.  The team-mode
   // wait for strip P - 1 is a warp-uniform spin on a shared-memory flag (a divergent spin makes
-  // every later shuffle take the slow diverged path).
+  // every later shuffle take the slow diverged path).  fcol = lane 0's column at that step.
   auto fetch = [&](int k, int fcol) {
-    ring_res[k] = cols[min(fcol, cmax)];
+    ring_res[k] = cols[min(fcol + 1, cmax)];
     if (from_prev) {
       const int rc = min(fcol, rlast);
       if constexpr (TEAM) {
@@ -265,15 +312,15 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
     }
   };
 #pragma unroll
-  for (int k = 0; k < 4; ++k) fetch(k, k);
+  for (int k = 0; k < 4; ++k) fetch(k, k - 1);
 
-  auto step = [&](auto kc, uint32_t* hin, uint32_t* hout) {
+  auto step = [&](auto kc) {
     constexpr int K = decltype(kc)::value;
     uint32_t x_hr = __shfl_up_sync(SWB_FULL, y_hr, 1, GC);
     uint32_t x_f = __shfl_up_sync(SWB_FULL, y_f, 1, GC);
     uint32_t x_res = __shfl_up_sync(SWB_FULL, y_res, 1, GC);
     if (gl == 0) { x_hr = ring_h[K]; x_f = ring_f[K]; x_res = ring_res[K]; }
-    // query-profile words for the two letters of this column
+    // query-profile words for the two letters of the NEXT column (look-ahead u)
     uint32_t wlo[R / 4], whi[R / 4];
     {
       const int alo = (x_res >> hshift) & 0xff;
@@ -283,48 +330,30 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
         load_prof<R, CB, GC * CB>(whi, prow + hi_off + ahi * ls);
       }
     }
-    fetch(K, col + gl + 4);   // lane 0's next column (col + gl is the step index)
-    // Vertical values travel as (H, F + rho) so that the F -> H -> F chain down the rows is
-    // two fused DPX ops per row: Fs = F + rho = max(Fs[i-1] - sigma, H[i-1]) and
-    // H = max(Fs - rho, u) with u = max(H[i-1][j-1] + w, E, 0) off the chain.
-    uint32_t hup = x_hr, fs = x_f, hprev = 0;
-    uint32_t hrdiag = hrdiag0;
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      e[r] = L::gap(e[r], nsig, hin[r]);                              // E = max(E[j-1] - sigma, H[j-1] - rho)
-      const uint32_t u = L::hcell(hrdiag, subst_row<L, R>(wlo, whi, r), e[r]);  // max(H[i-1][j-1] + w, E, 0)
-      fs = L::gap(fs, nsig, hup);                                     // F + rho = max(F[i-1] + rho - sigma, H[i-1])
-      const uint32_t h = L::gap(fs, nrho, u);                         // H = max(F, u)
-      hrdiag = hin[r];
-      hout[r] = L::add(h, nrho);                                      // H - rho (left value of the next column)
-      hup = h;
-      if (r & 1) best = L::max3(best, hprev, h); else hprev = h;
-    }
-    hrdiag0 = L::add(x_hr, nrho);
+    fetch(K, col + gl + 4);   // lane 0's column four steps on (col + gl + 1 is the step index)
+    uint32_t hup = x_hr, fs = x_f;
+    cell_rows<L, R>(e, u, wlo, whi, nrho, nsig, hup, fs, best);
     y_hr = hup; y_f = fs; y_res = x_res;
+    // keep the next step's residue shuffle (and so its profile loads) after this step's rows:
+    // hoisting them would keep a second set of profile words live (register spills at R = 44)
+    asm volatile("" : "+r"(y_res) : "r"(fs));
     // last lane: save the strip's bottom row for the next strip (not after the last strip);
-    // fill steps write neutral values that the real column overwrites later.  Team mode
-    // publishes progress every 16 columns (release: the row-buffer stores are visible first).
+    // fill steps write neutral values (index -1 keeps its neutral entry) that the real column
+    // overwrites later.  Team mode publishes progress every 16 columns (release: the row-buffer
+    // stores are visible first).
     if (store_out) {
-      rb_out[max(col, 0)] = make_uint2(y_hr, y_f);
+      rb_out[max(col, -1)] = make_uint2(y_hr, y_f);
       if (TEAM && col >= 0 && ((col & 15) == 15 || col == rlast)) st_release_smem(prog_out, pass_tag(P, col + 1));
     }
     ++col;
   };
 
-  // steps is a multiple of 4 (<= ncols + kPadCols); extra steps only see pad columns
+  // steps is a multiple of 4 (>= ncols + GC, <= ncols + kPadCols); extra steps only see pad columns
   for (int s = 0; s < steps; s += 4) {
-    if constexpr (PP) {
-      step(std::integral_constant<int, 0>{}, hrA, hrB);
-      step(std::integral_constant<int, 1>{}, hrB, hrA);
-      step(std::integral_constant<int, 2>{}, hrA, hrB);
-      step(std::integral_constant<int, 3>{}, hrB, hrA);
-    } else {
-      step(std::integral_constant<int, 0>{}, hrA, hrA);
-      step(std::integral_constant<int, 1>{}, hrA, hrA);
-      step(std::integral_constant<int, 2>{}, hrA, hrA);
-      step(std::integral_constant<int, 3>{}, hrA, hrA);
-    }
+    step(std::integral_constant<int, 0>{});
+    step(std::integral_constant<int, 1>{});
+    step(std::integral_constant<int, 2>{});
+    step(std::integral_constant<int, 3>{});
   }
   return best;
 }
@@ -369,7 +398,7 @@ __device__ __forceinline__ void emit(const SearchParams& p, uint32_t b, int pair
 // fetches it for the next strip at step T + len + 4 + j >= T + 52 + j (__syncwarp every group
 // in between).  A pair's score is reduced across the lanes once its last lane has moved on
 // (each lane parks its maximum in bdone when it leaves the pair's last strip).
-template <class L, int R, bool PP>
+template <class L, int R>
 __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainConst& c, const uint8_t* pbase,
                                              uint2* __restrict__ rb) {
   static_assert(R % 4 == 0, "R must be a multiple of 4");
@@ -378,7 +407,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
   const uint32_t nrho = L::splat(-c.rho);
   const uint32_t nsig = L::splat(-c.sigma);
   constexpr int CB = chunk_bytes<R>();
-  constexpr int kStripBytes = R * 32;          // (R / CB) chunks x 32 lanes x CB bytes
+  constexpr int kStripBytes = chunks_per_lane<R>() * 32 * CB;   // chunks x 32 lanes x CB bytes
   constexpr int kEndLen = 0xffffff;            // the END segment (after the last pair) never ends
   const int passes = p.short_passes;
   const int nshort = p.n_pairs - p.short_begin;
@@ -440,12 +469,15 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
       const uint32_t d = (uint32_t)f_len | ((uint32_t)(f_P + 1) << 24);
       if (f_seg & 1) desc1 = d; else desc0 = d;
     }
-    if (f_col < kGap || f_pair < 0) {   // gap: pad letters (the pair's trailing pad columns)
+    // residues one position ahead (look-ahead u, cell_rows): position f_col + k reads the
+    // letters of column f_col + k - kGap + 1; in the gap that is the pad column(s) stored just
+    // before the pair (kLeadCols / the previous pair's trailing pads), then its first column
+    if (f_pair < 0) {                   // END: pad letters (the last pair's trailing pad columns)
       g_cols = f_pad;
       g_rb = p.rb_zero;
     } else {
-      g_cols = f_cols + (f_col - kGap);
-      g_rb = f_P > 0 ? rb + (f_col - kGap) : p.rb_zero;
+      g_cols = f_cols + (f_col - kGap + 1);
+      g_rb = (f_col >= kGap && f_P > 0) ? rb + (f_col - kGap) : p.rb_zero;
     }
     if (f_pair >= 0) f_col += 4;
     fn += 4;
@@ -457,15 +489,10 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
     ring_h[k] = v.x; ring_f[k] = v.y;
   };
 
-  // ---- per-lane state
-  uint32_t hrA[R], hrB[PP ? R : 1], e[R];
+  // ---- per-lane state (look-ahead form, cell_rows)
+  uint32_t e[R], u[R];
 #pragma unroll
-  for (int r = 0; r < R; ++r) { hrA[r] = nrho; e[r] = nrho; }
-  if constexpr (PP) {
-#pragma unroll
-    for (int r = 0; r < R; ++r) hrB[r] = nrho;
-  }
-  uint32_t hrdiag0 = nrho;
+  for (int r = 0; r < R; ++r) { e[r] = nrho; u[r] = 0u; }
   uint32_t y_hr = 0, y_f = 0, y_res = c.padpair;
   uint32_t best = 0, bdone = 0;
   int my_pos = -lane, my_len = 0, my_P = -1, my_seg = -1;   // lane l reaches segment 0 at step l
@@ -476,31 +503,22 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
 #pragma unroll
   for (int k = 0; k < 4; ++k) fetch(k);
 
-  auto step = [&](auto kc, uint32_t* hin, uint32_t* hout) {
+  auto step = [&](auto kc) {
     constexpr int K = decltype(kc)::value;
     uint32_t x_hr = __shfl_up_sync(SWB_FULL, y_hr, 1);
     uint32_t x_f = __shfl_up_sync(SWB_FULL, y_f, 1);
     uint32_t x_res = __shfl_up_sync(SWB_FULL, y_res, 1);
     if (lane == 0) { x_hr = ring_h[K]; x_f = ring_f[K]; x_res = ring_res[K]; }
-    uint32_t wlo[R / 4], whi[R / 4];
+    uint32_t wlo[R / 4], whi[R / 4];   // profile words of the next position's letters
     load_prof<R, CB, 32 * CB>(wlo, prow + (x_res & 0xff) * ls);
     load_prof<R, CB, 32 * CB>(whi, prow + (x_res >> 8) * ls);
     fetch(K);
-    uint32_t hup = x_hr, fs = x_f, hprev = 0;
-    uint32_t hrdiag = hrdiag0;
-#pragma unroll
-    for (int r = 0; r < R; ++r) {   // the cell update of run_pass
-      e[r] = L::gap(e[r], nsig, hin[r]);
-      const uint32_t u = L::hcell(hrdiag, subst_row<L, R>(wlo, whi, r), e[r]);
-      fs = L::gap(fs, nsig, hup);
-      const uint32_t h = L::gap(fs, nrho, u);
-      hrdiag = hin[r];
-      hout[r] = L::add(h, nrho);
-      hup = h;
-      if (r & 1) best = L::max3(best, hprev, h); else hprev = h;
-    }
-    hrdiag0 = L::add(x_hr, nrho);
+    uint32_t hup = x_hr, fs = x_f;
+    cell_rows<L, R>(e, u, wlo, whi, nrho, nsig, hup, fs, best);
     y_hr = hup; y_f = fs; y_res = x_res;
+    // keep the next step's residue shuffle (and so its profile loads) after this step's rows:
+    // hoisting them would keep a second set of profile words live (register spills at R = 44)
+    asm volatile("" : "+r"(y_res) : "r"(fs));
     if (store_rb) {
       const int pos = my_pos + K;
       if (pos >= kGap && pos < my_len) rb[pos - kGap] = make_uint2(hup, fs);
@@ -520,8 +538,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
       store_rb = lane == 31 && my_P >= 0 && my_P < passes - 1;
       prow = pbase + max(my_P, 0) * kStripBytes;
 #pragma unroll
-      for (int r = 0; r < R; ++r) { hrA[r] = nrho; e[r] = nrho; }
-      hrdiag0 = nrho;
+      for (int r = 0; r < R; ++r) { e[r] = nrho; u[r] = 0u; }
     }
     __syncwarp();
     if (pending && S >= e_due) {   // every lane has parked the finished pair's maximum
@@ -533,17 +550,10 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
     }
     if (f_pair < 0 && !pending) break;
     plan_group();   // the 4 fetches issued during this group (consumed in the next one)
-    if constexpr (PP) {
-      step(std::integral_constant<int, 0>{}, hrA, hrB);
-      step(std::integral_constant<int, 1>{}, hrB, hrA);
-      step(std::integral_constant<int, 2>{}, hrA, hrB);
-      step(std::integral_constant<int, 3>{}, hrB, hrA);
-    } else {
-      step(std::integral_constant<int, 0>{}, hrA, hrA);
-      step(std::integral_constant<int, 1>{}, hrA, hrA);
-      step(std::integral_constant<int, 2>{}, hrA, hrA);
-      step(std::integral_constant<int, 3>{}, hrA, hrA);
-    }
+    step(std::integral_constant<int, 0>{});
+    step(std::integral_constant<int, 1>{});
+    step(std::integral_constant<int, 2>{});
+    step(std::integral_constant<int, 3>{});
     my_pos += 4;
   }
 }
@@ -614,13 +624,13 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
         // P + W before all its lanes finished strip P: its lane 0 may wait for strip P + W - 1,
         // which transitively needs the tail of strip P (deadlock for short rows otherwise).
         uint32_t b = 0;
-        const int tsteps = (ncols + 31 + 3) & ~3;
+        const int tsteps = (ncols + 32 + 3) & ~3;
         for (int P = wt; P < p.long_passes; P += W) {
           const int si = (P + W) % (W + 1), so = P % (W + 1);   // slot of strip P-1 / strip P
           constexpr int CBl = chunk_bytes<Rl>();
-          const uint8_t* prow = smem + p.lt.off + (P * (Rl / CBl) * 32 + lane) * CBl;
-          b = run_pass<L, 32, Rl, true, PP>(c, prow, p.lt.ls, 0, cp, ncols, half, tsteps, P, p.long_passes,
-                                        rb + (int64_t)si * p.rb_team_cols, rb + (int64_t)so * p.rb_team_cols,
+          const uint8_t* prow = smem + p.lt.off + (P * chunks_per_lane<Rl>() * 32 + lane) * CBl;
+          b = run_pass<L, 32, Rl, true>(c, prow, p.lt.ls, 0, cp, ncols, half, tsteps, P, p.long_passes,
+                                        rb + (int64_t)si * p.rb_team_cols + 1, rb + (int64_t)so * p.rb_team_cols + 1,
                                         prog + si, prog + so, b);
         }
 #pragma unroll
@@ -640,7 +650,7 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
   if constexpr (G == 32) {
     if (p.item_list == nullptr && p.group_stream) {
       constexpr int CBs = chunk_bytes<Rs>();
-      group_stream<L, Rs, PP>(p, c, smem + p.lg.off + lane * CBs,
+      group_stream<L, Rs>(p, c, smem + p.lg.off + lane * CBs,
                               p.rb_group + (int64_t)(blockIdx.x * kWarps + warp) * p.rb_group_cols);
       return;
     }
@@ -658,13 +668,13 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
       const int pair = p.short_begin + base + gi;
       const int ncols = valid ? p.pair_ncols[pair] : 0;
       const uint16_t* cp = p.cols + (valid ? p.pair_off[pair] : 0);
-      const int steps = ((int)__reduce_max_sync(SWB_FULL, (unsigned)ncols) + G - 1 + 3) & ~3;
+      const int steps = ((int)__reduce_max_sync(SWB_FULL, (unsigned)ncols) + G + 3) & ~3;
       uint2* rb = p.rb_group + ((int64_t)(blockIdx.x * kWarps + warp) * GPW + gi) * p.rb_group_cols;
       uint32_t b = 0;
       for (int P = 0; P < p.short_passes; ++P) {
         constexpr int CBs = chunk_bytes<Rs>();
-        const uint8_t* prow = smem + p.lg.off + gi * p.lg.rs + (P * (Rs / CBs) * G + gl) * CBs;
-        b = run_pass<L, G, Rs, false, PP>(c, prow, p.lg.ls, 0, cp, ncols, 0, steps, P, p.short_passes, rb, rb, nullptr,
+        const uint8_t* prow = smem + p.lg.off + gi * p.lg.rs + (P * chunks_per_lane<Rs>() * G + gl) * CBs;
+        b = run_pass<L, G, Rs, false>(c, prow, p.lg.ls, 0, cp, ncols, 0, steps, P, p.short_passes, rb + 1, rb + 1, nullptr,
                                       nullptr, b);
         __syncwarp();   // strip P's bottom row (written by lane G-1) is read by lane 0 in strip P+1
       }
@@ -701,7 +711,7 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const ChainConst& 
   constexpr int LS = 32 * C;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int A1 = p.A + 1;
-  const int qsteps = (p.qcols + 31 + 3) & ~3;
+  const int qsteps = (p.qcols + 32 + 3) & ~3;
   int pending = first_item;
   for (;;) {
     team_bar(team, W);
@@ -750,8 +760,8 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const ChainConst& 
       }
       __syncwarp();
       const int si = (P + W) % (W + 1), so = P % (W + 1);
-      b = run_pass<L, 32, C, true, PP>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps, P, S,
-                                       rb + (int64_t)si * p.rb_cols, rb + (int64_t)so * p.rb_cols, prog + si,
+      b = run_pass<L, 32, C, true>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps, P, S,
+                                       rb + (int64_t)si * p.rb_cols + 1, rb + (int64_t)so * p.rb_cols + 1, prog + si,
                                        prog + so, b);
     }
 #pragma unroll

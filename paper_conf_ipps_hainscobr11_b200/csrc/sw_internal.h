@@ -10,12 +10,17 @@ constexpr int kMaxWarps = 16;            // at most 512 threads per CTA
 constexpr int kMinCols = 48;             // every pair is padded to >= 48 columns (>= G + 16)
 constexpr int kColAlign = 8;             // pair column counts are multiples of 8 (16 bytes)
 constexpr int kPadCols = 32;             // trailing pad columns stored after every pair
+constexpr int kLeadCols = 8;             // pad columns stored before the first pair, so that every
+                                         // pair is preceded by >= 3 pad columns (the look-ahead
+                                         // residue stream of group_stream reads them)
 constexpr int kPadValue = -128;          // profile value of pad letters / pad query rows
 
 // Bank-conflict-free shared-memory image of the query profile for chains of G lanes with R
 // rows per lane.  Query row i lives in strip P = i / (G*R),
 // lane gl = (i % (G*R)) / R, row r = i % R, chunk k = r / cb (cb = 4 or 8 rows = bytes):
-//   byte(rep, a, i) = off + rep*rs + a*ls + ((P*(R/cb) + k)*G + gl)*cb + r % cb
+//   byte(rep, a, i) = off + rep*rs + a*ls + ((P*nch + k)*G + gl)*cb + r % cb
+// (nch = ceil(R / cb) chunks per lane and strip; cb = 16 from 12 rows up, the last chunk
+// partial when R % 16 != 0: LDS.128 reads 4 query rows x 4 per instruction)
 // so at a fixed (strip, chunk) the G lanes of a chain read consecutive cb-byte words of
 // their own letter row: the letter term a*ls is a multiple of 128 B (32 banks) and drops
 // out of the bank index, and the 32/G replicas (one per chain of a warp) are shifted by
@@ -25,6 +30,7 @@ struct ProfLayout {
   int G;       // lanes per chain (32 for team mode)
   int R;       // rows per lane
   int cb;      // chunk bytes
+  int nch;     // chunks per lane and strip, ceil(R / cb)
   int strips;  // strips covered (strips * G * R >= m)
   int ls;      // letter stride, multiple of 128
   int rs;      // replica stride, == cb * G (mod 128)

@@ -22,7 +22,7 @@ __global__ void k_profile(uint8_t* __restrict__ blob, const ProfLayout L, const 
     const int rep = (int)(t / ((int64_t)rows * (A + 1)));
     const int P = i / (L.G * L.R), qq = i % (L.G * L.R), gl = qq / L.R, r = qq % L.R;
     const int64_t addr = (int64_t)L.off + (int64_t)rep * L.rs + (int64_t)a * L.ls +
-                         ((int64_t)(P * (L.R / L.cb) + r / L.cb) * L.G + gl) * L.cb + r % L.cb;
+                         ((int64_t)(P * L.nch + r / L.cb) * L.G + gl) * L.cb + r % L.cb;
     int v = kPadValue;
     if (a < A && i < m) v = (int)W[q[i] * A + a] + rho;
     blob[addr] = (uint8_t)(int8_t)v;
