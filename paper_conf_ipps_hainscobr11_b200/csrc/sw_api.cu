@@ -147,7 +147,8 @@ int cuda_fail(sw_handle h, cudaError_t e, const char* what) {
   } while (0)
 
 template <class T>
-int grow(sw_handle h, T** p, size_t* cap, size_t bytes, const char* what, cudaStream_t busy = nullptr) {
+int grow(sw_handle h, T** p, size_t* cap, size_t bytes, const char* what, cudaStream_t busy = nullptr,
+         bool zero = false) {
   if (*cap >= bytes && *p) return SW_OK;
   if (busy) cudaStreamSynchronize(busy);  // the old buffer may still be in use on this stream
   if (*p) cudaFree(*p);
@@ -156,10 +157,13 @@ int grow(sw_handle h, T** p, size_t* cap, size_t bytes, const char* what, cudaSt
   if (bytes == 0) return SW_OK;
   cudaError_t e = cudaMalloc(reinterpret_cast<void**>(p), bytes);
   if (e != cudaSuccess) return cuda_fail(h, e, what);
-  // zero-filled: the row buffers' leading slot of every strip buffer must read as the neutral
-  // entry (H, F + rho) = (0, 0) (run_pass); it is only ever rewritten with neutral values
-  e = busy ? cudaMemsetAsync(*p, 0, bytes, busy) : cudaMemset(*p, 0, bytes);
-  if (e != cudaSuccess) return cuda_fail(h, e, what);
+  // zero: the row buffers' leading slot of every strip buffer must read as the neutral entry
+  // (H, F + rho) = (0, 0) (run_pass); it is only ever rewritten with neutral values.  Ordered
+  // on the stream that will use the buffer.
+  if (zero) {
+    e = cudaMemsetAsync(*p, 0, bytes, busy);
+    if (e != cudaSuccess) return cuda_fail(h, e, what);
+  }
   *cap = bytes;
   return SW_OK;
 }
@@ -446,9 +450,9 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
     const int nteams = (pl.rcfg.threads / 32) / pl.r_team_warps;
     rbt = std::max(rbt, (size_t)pl.rgrid * nteams * (pl.r_team_warps + 1) * max_cols_all * sizeof(uint2));
   }
-  rc = grow(h, &s.d_rb_group, &s.rb_group_cap, rbg, "alloc group row buffers", s.stream);
+  rc = grow(h, &s.d_rb_group, &s.rb_group_cap, rbg, "alloc group row buffers", s.stream, true);
   if (rc) return rc;
-  rc = grow(h, &s.d_rb_team, &s.rb_team_cap, rbt, "alloc team row buffers", s.stream);
+  rc = grow(h, &s.d_rb_team, &s.rb_team_cap, rbt, "alloc team row buffers", s.stream, true);
   if (rc) return rc;
 
   const int qcols = (int)round_up(m, 8);
@@ -467,7 +471,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
               s.stream);
     if (rc) return rc;
     rc = grow(h, &s.d_rb_t, &s.rb_t_cap, (size_t)t_grid * 2 * t_warps * (qcols + kPadCols + 1) * sizeof(uint2),
-              "alloc long-sequence row buffers", s.stream);
+              "alloc long-sequence row buffers", s.stream, true);
     if (rc) return rc;
   }
 

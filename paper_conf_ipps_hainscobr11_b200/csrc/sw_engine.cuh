@@ -154,17 +154,18 @@ __device__ __forceinline__ void team_bar(int team, int W) {
 // chunks of CB bytes, STRIDE bytes apart (ProfLayout); with CB = 16 the last chunk may be
 // partial (R % 16 rows), read with the narrowest load that covers it.
 template <int R, int CB, int STRIDE>
-__device__ __forceinline__ void load_prof(uint32_t (&w)[R / 4], const uint8_t* p) {
+__device__ __forceinline__ void load_prof(uint32_t (&w)[(R + 3) / 4], const uint8_t* p) {
   if constexpr (CB == 16) {
 #pragma unroll
     for (int k = 0; k < R / 16; ++k) {
       const uint4 v = *reinterpret_cast<const uint4*>(p + k * STRIDE);
       w[4 * k + 0] = v.x; w[4 * k + 1] = v.y; w[4 * k + 2] = v.z; w[4 * k + 3] = v.w;
     }
-    constexpr int k = R / 16, rem = (R % 16) / 4;
-    if constexpr (rem == 3) {
+    constexpr int k = R / 16, rem = (R % 16 + 3) / 4;   // words of the partial chunk
+    if constexpr (rem >= 3) {
       const uint4 v = *reinterpret_cast<const uint4*>(p + k * STRIDE);
       w[4 * k + 0] = v.x; w[4 * k + 1] = v.y; w[4 * k + 2] = v.z;
+      if constexpr (rem == 4) w[4 * k + 3] = v.w;
     } else if constexpr (rem == 2) {
       const uint2 v = *reinterpret_cast<const uint2*>(p + k * STRIDE);
       w[4 * k + 0] = v.x; w[4 * k + 1] = v.y;
@@ -193,7 +194,7 @@ __host__ __device__ constexpr int chunks_per_lane() { return (R + chunk_bytes<R>
 
 // substitution value (w + rho) of row r of the lane's window, packed per Lane
 template <class L, int R>
-__device__ __forceinline__ uint32_t subst_row(const uint32_t (&wlo)[R / 4], const uint32_t (&whi)[R / 4], int r) {
+__device__ __forceinline__ uint32_t subst_row(const uint32_t (&wlo)[(R + 3) / 4], const uint32_t (&whi)[(R + 3) / 4], int r) {
   const uint32_t a = wlo[r >> 2];
   const uint32_t b = (L::kSeqs == 2) ? whi[r >> 2] : 0u;
   switch (r & 3) {
@@ -228,8 +229,8 @@ struct ChainConst {
 //   best = max(best, h, h') every two rows                         VIMNMX3
 // plus one PRMT per row for w + rho of column j+1 (profile words of the next column's letters).
 template <class L, int R>
-__device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&u)[R], const uint32_t (&wlo)[R / 4],
-                                          const uint32_t (&whi)[R / 4], uint32_t nrho, uint32_t nsig,
+__device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&u)[R], const uint32_t (&wlo)[(R + 3) / 4],
+                                          const uint32_t (&whi)[(R + 3) / 4], uint32_t nrho, uint32_t nsig,
                                           uint32_t& hup, uint32_t& fs, uint32_t& best) {
   uint32_t hrup = L::add(hup, nrho), hprev = 0;
 #pragma unroll
@@ -243,6 +244,7 @@ __device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&u)[R], co
     hup = h;
     if (r & 1) best = L::max3(best, hprev, h); else hprev = h;
   }
+  if constexpr (R & 1) best = L::max2(best, hprev);
 }
 
 // One strip pass of a chain of GC lanes over the columns of one database pair (see the file
@@ -261,7 +263,7 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
                                              int half, int steps, int P, int passes_total,
                                              const uint2* __restrict__ rb_in, uint2* __restrict__ rb_out,
                                              const uint32_t* prog_in, uint32_t* prog_out, uint32_t best) {
-  static_assert(R % 4 == 0, "R must be a multiple of 4");
+  static_assert(R % 4 == 0 || R >= 12, "R < 12 must be a multiple of 4");
   const int lane = threadIdx.x & 31;
   const int gl = lane & (GC - 1);
   const uint32_t nrho = L::splat(-c.rho);
@@ -321,7 +323,7 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
     uint32_t x_res = __shfl_up_sync(SWB_FULL, y_res, 1, GC);
     if (gl == 0) { x_hr = ring_h[K]; x_f = ring_f[K]; x_res = ring_res[K]; }
     // query-profile words for the two letters of the NEXT column (look-ahead u)
-    uint32_t wlo[R / 4], whi[R / 4];
+    uint32_t wlo[(R + 3) / 4], whi[(R + 3) / 4];
     {
       const int alo = (x_res >> hshift) & 0xff;
       load_prof<R, CB, GC * CB>(wlo, prow + alo * ls);
@@ -401,7 +403,7 @@ __device__ __forceinline__ void emit(const SearchParams& p, uint32_t b, int pair
 template <class L, int R>
 __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainConst& c, const uint8_t* pbase,
                                              uint2* __restrict__ rb) {
-  static_assert(R % 4 == 0, "R must be a multiple of 4");
+  static_assert(R % 4 == 0 || R >= 12, "R < 12 must be a multiple of 4");
   constexpr int kGap = 4;
   const int lane = threadIdx.x & 31;
   const uint32_t nrho = L::splat(-c.rho);
@@ -509,7 +511,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
     uint32_t x_f = __shfl_up_sync(SWB_FULL, y_f, 1);
     uint32_t x_res = __shfl_up_sync(SWB_FULL, y_res, 1);
     if (lane == 0) { x_hr = ring_h[K]; x_f = ring_f[K]; x_res = ring_res[K]; }
-    uint32_t wlo[R / 4], whi[R / 4];   // profile words of the next position's letters
+    uint32_t wlo[(R + 3) / 4], whi[(R + 3) / 4];   // profile words of the next position's letters
     load_prof<R, CB, 32 * CB>(wlo, prow + (x_res & 0xff) * ls);
     load_prof<R, CB, 32 * CB>(whi, prow + (x_res >> 8) * ls);
     fetch(K);
@@ -558,7 +560,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
   }
 }
 
-template <class L, int G, int Rs, int Rl, int NT, bool PP>
+template <class L, int G, int Rs, int Rl, int NT>
 __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
   constexpr int kWarps = NT / 32;
   extern __shared__ __align__(128) uint8_t smem[];
@@ -701,7 +703,7 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
 // an item already taken for this team (or -1).  max_strips: a team of W warps only keeps items
 // with at most this many strips (> max_strips: the item is parked in *parked and the loop
 // returns, so that the CTA can regroup into smaller teams for the remaining, shorter items).
-template <int C, bool PP>
+template <int C>
 __device__ __forceinline__ void t_team_loop(const TParams& p, const ChainConst& c, uint8_t* tab,
                                             const int8_t* wp, int W, int team, int wt, int first_item,
                                             int min_strips, int* parked, uint32_t* prog, uint2* rb,
@@ -782,7 +784,7 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const ChainConst& 
   }
 }
 
-template <int C, int NT, bool PP>
+template <int C, int NT>
 __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   constexpr int kWarps = NT / 32;
   constexpr int LS = 32 * C;
@@ -816,7 +818,7 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   // Phase 2: teams of team_warps for the rest — small teams waste less time in the pipeline
   // fill and in the end-of-item barrier (T-mode ncu: 17 % barrier stalls with 8-warp teams).
   if (p.warps > p.team_warps) {
-    t_team_loop<C, PP>(p, c, tab, wp, p.warps, 0, warp, -1, p.big_strips, &sparked, sprog, rb_cta, sitem, sred);
+    t_team_loop<C>(p, c, tab, wp, p.warps, 0, warp, -1, p.big_strips, &sparked, sprog, rb_cta, sitem, sred);
     __syncthreads();
   }
   const int W = p.team_warps;
@@ -824,36 +826,36 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   const int team = warp / W, wt = warp % W;
   if (team >= nteams) return;
   const int first = (team == 0) ? sparked : -1;
-  t_team_loop<C, PP>(p, c, tab, wp, W, team, wt, first, 0, nullptr, sprog + team * (W + 1),
+  t_team_loop<C>(p, c, tab, wp, W, team, wt, first, 0, nullptr, sprog + team * (W + 1),
                      rb_cta + (int64_t)team * (W + 1) * p.rb_cols, sitem, sred);
 }
 
-template <int C, int NT, bool PP>
+template <int C, int NT>
 cudaError_t launch_search_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st) {
-  k_search_t<C, NT, PP><<<grid, NT, smem_bytes, st>>>(p);
+  k_search_t<C, NT><<<grid, NT, smem_bytes, st>>>(p);
   return cudaGetLastError();
 }
 
-template <int C, int NT, bool PP>
+template <int C, int NT>
 cudaError_t configure_tmode(int smem_bytes, int* blocks_per_sm) {
   cudaError_t e =
-      cudaFuncSetAttribute(k_search_t<C, NT, PP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+      cudaFuncSetAttribute(k_search_t<C, NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search_t<C, NT, PP>, NT, smem_bytes);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search_t<C, NT>, NT, smem_bytes);
 }
 
-template <class L, int G, int Rs, int Rl, int NT, bool PP>
+template <class L, int G, int Rs, int Rl, int NT>
 cudaError_t launch_search_t(const SearchParams& p, int grid, int smem_bytes, cudaStream_t st) {
-  k_search<L, G, Rs, Rl, NT, PP><<<grid, NT, smem_bytes, st>>>(p);
+  k_search<L, G, Rs, Rl, NT><<<grid, NT, smem_bytes, st>>>(p);
   return cudaGetLastError();
 }
 
-template <class L, int G, int Rs, int Rl, int NT, bool PP>
+template <class L, int G, int Rs, int Rl, int NT>
 cudaError_t configure_t(int smem_bytes, int* blocks_per_sm) {
-  cudaError_t e = cudaFuncSetAttribute(k_search<L, G, Rs, Rl, NT, PP>,
+  cudaError_t e = cudaFuncSetAttribute(k_search<L, G, Rs, Rl, NT>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search<L, G, Rs, Rl, NT, PP>, NT,
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search<L, G, Rs, Rl, NT>, NT,
                                                        smem_bytes);
 }
 

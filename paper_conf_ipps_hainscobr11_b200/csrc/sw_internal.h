@@ -85,7 +85,6 @@ struct KernelConfig {
   int Rs;
   int Rl;
   int threads;   // CTA size (fewer threads for the register-heavy entries)
-  int pingpong;  // 1: two register arrays for H - rho (see run_pass)
 };
 
 // Launch one search; returns the CUDA error of the launch.

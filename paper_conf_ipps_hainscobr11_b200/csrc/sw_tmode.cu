@@ -19,11 +19,11 @@ cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, int pad,
 }
 
 cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st) {
-  return launch_search_tmode<kTmodeC, kTmodeThreads, true>(p, grid, smem_bytes, st);
+  return launch_search_tmode<kTmodeC, kTmodeThreads>(p, grid, smem_bytes, st);
 }
 
 cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm) {
-  return configure_tmode<kTmodeC, kTmodeThreads, true>(smem_bytes, blocks_per_sm);
+  return configure_tmode<kTmodeC, kTmodeThreads>(smem_bytes, blocks_per_sm);
 }
 
 }  // namespace swb

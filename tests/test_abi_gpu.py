@@ -139,6 +139,22 @@ def test_search_stream_matches_oracle(chunk):
             assert np.array_equal(outb[k], oracle.scores(qq, BLOSUM62, 10, 2, db.residues, db.offsets))
 
 
+def test_search_stream_growing_chunks_match_resident():
+    """Chunks of growing size force the device database buffers of a stream slot to be
+    reallocated while the other slot's search runs: the streamed scores must equal the
+    resident search bit for bit (regression: a zero-fill of freshly allocated buffers on the
+    legacy stream raced the upload stream and corrupted chunks)."""
+    lens = gen.sp_lengths(60_000, seed=21)
+    lens[::7] += np.arange(lens[::7].size) % 700            # later chunks hold longer sequences
+    db = gen.build_database(np.sort(lens), 21)
+    q = gen.make_query(5478)
+    with swp.SmithWaterman(q, BLOSUM62, 10, 2) as sw:
+        sw.load_db(db.residues, db.offsets)
+        ref = sw.search(3072)
+        for chunk in (1 << 20, 3 << 20):
+            assert np.array_equal(sw.search_stream(db.residues, db.offsets, 3072, chunk).reshape(-1), ref)
+
+
 def test_search_stream_errors_and_empty():
     L = swp.load_library()
     with swp.SmithWaterman(gen.make_query(40), BLOSUM62, 10, 2) as sw:
