@@ -290,38 +290,42 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
   // (bounded, legitimate DP values of the extended matrix).
   const int cmax = ncols + kPadCols - 1;
   const int rlast = steps - GC - 1;
-  uint32_t ring_res[4], ring_h[4], ring_f[4];   // top boundary: H[0][j] = 0, F[0][j] + rho <= 0
+  // two 4-deep rings (A: this group's steps, B: the next group's), top boundary H[0][j] = 0,
+  // F[0][j] + rho <= 0 when there is no previous strip
+  uint32_t rrA[4], rhA[4], rfA[4], rrB[4], rhB[4], rfB[4];
 #pragma unroll
-  for (int k = 0; k < 4; ++k) { ring_res[k] = c.padpair; ring_h[k] = 0; ring_f[k] = 0; }
+  for (int k = 0; k < 4; ++k) { rhA[k] = rfA[k] = rhB[k] = rfB[k] = 0; rrA[k] = rrB[k] = c.padpair; }
   uint32_t known = 0;   // team mode: last progress value seen for strip P - 1
   // Every lane of the chain runs the fetch (same addresses as its lane 0: broadcast loads, no
-  // extra traffic) so the warp never diverges; only lane 0 consumes the values.  The team-mode
-  // wait for strip P - 1 is a warp-uniform spin on a shared-memory flag (a divergent spin makes
-  // every later shuffle take the slow diverged path).  fcol = lane 0's column at that step.
-  auto fetch = [&](int k, int fcol) {
-    ring_res[k] = cols[min(fcol + 1, cmax)];
+  // extra traffic) so the warp never diverges; only lane 0 consumes the values.  One fetch per
+  // group of 4 steps (lane-0 columns c0 .. c0 + 3), one team-mode wait per group: a
+  // warp-uniform spin on a shared-memory flag (a divergent spin makes every later shuffle take
+  // the slow diverged path).
+  auto fetch_group = [&](uint32_t (&rr)[4], uint32_t (&rh)[4], uint32_t (&rf)[4], int c0) {
+#pragma unroll
+    for (int k = 0; k < 4; ++k) rr[k] = cols[min(c0 + k + 1, cmax)];
     if (from_prev) {
-      const int rc = min(fcol, rlast);
       if constexpr (TEAM) {
-        const uint32_t need = pass_tag(P - 1, rc + 1);
+        const uint32_t need = pass_tag(P - 1, min(c0 + 3, rlast) + 1);
         while (known < need) {
           known = ld_acquire_smem(prog_in);
           if (known < need) __nanosleep(32);
         }
       }
-      const uint2 v = rb_in[rc];
-      ring_h[k] = v.x; ring_f[k] = v.y;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const uint2 v = rb_in[min(c0 + k, rlast)];
+        rh[k] = v.x; rf[k] = v.y;
+      }
     }
   };
-#pragma unroll
-  for (int k = 0; k < 4; ++k) fetch(k, k - 1);
 
-  auto step = [&](auto kc) {
+  auto step = [&](auto kc, const uint32_t (&rr)[4], const uint32_t (&rh)[4], const uint32_t (&rf)[4]) {
     constexpr int K = decltype(kc)::value;
     uint32_t x_hr = __shfl_up_sync(SWB_FULL, y_hr, 1, GC);
     uint32_t x_f = __shfl_up_sync(SWB_FULL, y_f, 1, GC);
     uint32_t x_res = __shfl_up_sync(SWB_FULL, y_res, 1, GC);
-    if (gl == 0) { x_hr = ring_h[K]; x_f = ring_f[K]; x_res = ring_res[K]; }
+    if (gl == 0) { x_hr = rh[K]; x_f = rf[K]; x_res = rr[K]; }
     // query-profile words for the two letters of the NEXT column (look-ahead u)
     uint32_t wlo[(R + 3) / 4], whi[(R + 3) / 4];
     {
@@ -332,30 +336,42 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
         load_prof<R, CB, GC * CB>(whi, prow + hi_off + ahi * ls);
       }
     }
-    fetch(K, col + gl + 4);   // lane 0's column four steps on (col + gl + 1 is the step index)
     uint32_t hup = x_hr, fs = x_f;
     cell_rows<L, R>(e, u, wlo, whi, nrho, nsig, hup, fs, best);
     y_hr = hup; y_f = fs; y_res = x_res;
-    // keep the next step's residue shuffle (and so its profile loads) after this step's rows:
-    // hoisting them would keep a second set of profile words live (register spills at R = 44)
-    asm volatile("" : "+r"(y_res) : "r"(fs));
     // last lane: save the strip's bottom row for the next strip (not after the last strip);
     // fill steps write neutral values (index -1 keeps its neutral entry) that the real column
-    // overwrites later.  Team mode publishes progress every 16 columns (release: the row-buffer
-    // stores are visible first).
-    if (store_out) {
-      rb_out[max(col, -1)] = make_uint2(y_hr, y_f);
-      if (TEAM && col >= 0 && ((col & 15) == 15 || col == rlast)) st_release_smem(prog_out, pass_tag(P, col + 1));
-    }
+    // overwrites later.
+    if (store_out) rb_out[max(col, -1)] = make_uint2(y_hr, y_f);
     ++col;
   };
+  // team mode: publish this strip's progress when a group crossed a multiple of 16 columns or
+  // reached the last one (release: the row-buffer stores are visible first)
+  auto publish = [&]() {
+    if (TEAM && store_out) {
+      const int done = col;   // the last lane's columns < col are stored
+      if (done > 0 && ((done & 15) < 4 || done > rlast))
+        st_release_smem(prog_out, pass_tag(P, min(done, rlast + 1)));
+    }
+  };
 
-  // steps is a multiple of 4 (>= ncols + GC, <= ncols + kPadCols); extra steps only see pad columns
-  for (int s = 0; s < steps; s += 4) {
-    step(std::integral_constant<int, 0>{});
-    step(std::integral_constant<int, 1>{});
-    step(std::integral_constant<int, 2>{});
-    step(std::integral_constant<int, 3>{});
+  // steps is a multiple of 4 (>= ncols + GC, <= ncols + kPadCols); extra steps only see pad
+  // columns.  Lane 0's column at step s is s - 1.
+  fetch_group(rrA, rhA, rfA, -1);
+  for (int s = 0; s < steps; s += 8) {
+    fetch_group(rrB, rhB, rfB, s + 3);
+    step(std::integral_constant<int, 0>{}, rrA, rhA, rfA);
+    step(std::integral_constant<int, 1>{}, rrA, rhA, rfA);
+    step(std::integral_constant<int, 2>{}, rrA, rhA, rfA);
+    step(std::integral_constant<int, 3>{}, rrA, rhA, rfA);
+    publish();
+    if (s + 4 >= steps) break;
+    fetch_group(rrA, rhA, rfA, s + 7);
+    step(std::integral_constant<int, 0>{}, rrB, rhB, rfB);
+    step(std::integral_constant<int, 1>{}, rrB, rhB, rfB);
+    step(std::integral_constant<int, 2>{}, rrB, rhB, rfB);
+    step(std::integral_constant<int, 3>{}, rrB, rhB, rfB);
+    publish();
   }
   return best;
 }
