@@ -206,6 +206,7 @@ struct Plan {
   int grid, rgrid;
   double cost;         // estimated cycles of the main launch
   double thr, tail_s;  // its throughput term and the critical path of the longest short item
+  double thr_full;     // the throughput term at full occupancy (no few-items penalty)
 };
 
 int team_warps_for(int passes, int warps) {
@@ -269,11 +270,12 @@ int make_plan(sw_handle h, int m, const Split& sp, Plan* pl) {
     double thr = (gsteps * is + tsteps * il) / kGpuIssue;
     // few items: the issue rate needs ~2 busy warps per scheduler (4 per SM)
     const double active_warps = (double)sp.n_short / (32 / c.G) + (double)sp.n_long * W;
+    const double thr_full = thr;
     thr /= std::min(1.0, std::max(0.05, active_warps / (8.0 * h->num_sms)));
     const double tail_l = sp.n_long ? (sp.long_max_cols + 31.0) * ((lt.strips + W - 1) / W) * il / kWarpIssue : 0.0;
     const double tail_s = sp.n_short ? (sp.short_max_cols + c.G - 1.0) * lg.strips * is / kWarpIssue : 0.0;
     const double cost = std::max(thr, std::max(tail_l, tail_s));
-    if (cost < best) { best = cost; best_i = i; pl->thr = thr; pl->tail_s = tail_s; }
+    if (cost < best) { best = cost; best_i = i; pl->thr = thr; pl->tail_s = tail_s; pl->thr_full = thr_full; }
   }
   pl->cost = best;
   // test hooks: force a menu entry / team size (used by the parity tests to cover every
@@ -373,8 +375,16 @@ int64_t choose_threshold(sw_handle h, int m) {
   {
     Split sp = make_split(h, maxlen + 1, nullptr);
     Plan pl;
-    if (!make_plan(h, m, sp, &pl) && sp.short_cols > 0) per_col = pl.thr * (2.7 / 2.0) / (double)sp.short_cols;
+    if (!make_plan(h, m, sp, &pl) && sp.short_cols > 0) per_col = pl.thr_full * (2.7 / 2.0) / (double)sp.short_cols;
   }
+  // long path cost per column relative to the group path at full occupancy, measured (C3 all
+  // long vs C2 short, profiles/r01_sweep_c3_*.jsonl): 2.4 at m = 144, 1.57 at 567, 1.43 at
+  // 1500, 1.21 at 5478 (linear in between)
+  const double lm[] = {144, 567, 1500, 5478}, lf[] = {2.4, 1.57, 1.43, 1.21};
+  double long_factor = lf[3];
+  if (m <= lm[0]) long_factor = lf[0];
+  for (int k = 0; k < 3; ++k)
+    if (m > lm[k] && m <= lm[k + 1]) long_factor = lf[k] + (lf[k + 1] - lf[k]) * (m - lm[k]) / (lm[k + 1] - lm[k]);
   for (int64_t T : cands) {
     if (T > maxlen + 1) continue;
     Split sp = make_split(h, T, nullptr);
@@ -386,7 +396,7 @@ int64_t choose_threshold(sw_handle h, int m) {
     // measured rates: the whole GPU sustains ~0.5 ALU warp-instructions / clock / scheduler
     // (not the model's 2.7 / SM), and a tail warp ~0.15 (profiles/r01_ncu_*, query sweeps)
     const double thr = pl.thr * (2.7 / 2.0), tail = pl.tail_s * (0.2 / 0.15);
-    const double thr_long = per_col * long_cols * 1.8;
+    const double thr_long = per_col * long_cols * long_factor;
     const double cost = std::max(thr + thr_long, tail / 0.8);
     if (getenv("SW_DEBUG_AUTO"))
       fprintf(stderr, "auto m=%d T=%lld G=%d Rs=%d thr=%.3f long=%.3f tail=%.3f cost=%.3f ms\n", m, (long long)T,
@@ -410,8 +420,10 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   if (rc) return rc;
   // Long pairs: T-mode (strips along the database sequence) when the query is short enough
   // that team mode would have few query strips to spread over warps; team mode otherwise.
-  // SW_LONG_MODE=team|t overrides (tests).
-  bool use_t = n_long > 0 && pl.long_passes <= 2;
+  // Measured on C3 (all long, profiles/r01_longmode_grid.txt): T-mode ahead up to m = 2504
+  // (567: 3347 vs 1190 GCUPS, 1500: 3676 vs 2655, 2504: 3765 vs 3507), team mode from
+  // m = 3564 (3916 vs 3795, 5478: 4335 vs 3838).  SW_LONG_MODE=team|t overrides (tests).
+  bool use_t = n_long > 0 && m < kTmodeMaxQuery;
   if (const char* f = getenv("SW_LONG_MODE")) {
     if (!strcmp(f, "team")) use_t = false;
     if (!strcmp(f, "t")) use_t = n_long > 0;
@@ -543,17 +555,48 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
     t.ovf_count = s.d_ovf_count;
     t.work = s.d_work + 3;
     t.warps = t_warps;
-    // Phase 1: pairs with >= big_strips strips (8192 positions) take the whole CTA as one
-    // team; phase 2: teams of W warps, W ~ a quarter of a typical pair's strips (fill and
-    // end-of-item waits grow as W^2 / strips), W in {1, 2, 4, 8}, W | t_warps.
-    const double avg_strips = (double)sp.long_cols / std::max(1, n_long) / (32.0 * kTmodeC);
-    int W = 1;
-    while (W * 2 <= t_warps && W * 2 <= avg_strips / 4.0 + 0.5 && t_warps % (W * 2) == 0) W *= 2;
-    if (const char* f = getenv("SW_T_TEAM")) W = std::max(1, std::min(t_warps, atoi(f)));
-    while (t_warps % W) --W;
-    t.team_warps = W;
-    t.big_strips = 16;
-    if (const char* f = getenv("SW_T_BIG")) t.big_strips = std::max(1, atoi(f));
+    // Team sizes from a time model.  A team of W warps walks
+    // the S strips of a pair; strip s + 1 trails strip s by ~lag steps (32-lane fill + the
+    // 16-column progress granularity), each strip is qsteps = m + 32 steps, so a team is
+    // pipeline-bound unless W * lag <= qsteps.  Phase 1 (pairs with >= big_strips strips, one
+    // team of all t_warps warps) only pays when the longest pair's time dominates.
+    //   est = max(sum over phases of warp-steps / (all warps x utilisation), longest pair)
+    {
+      const double lag = 44.0, qsteps = (double)round_up(qcols + 32, 4);
+      const double nw = (double)t_grid * t_warps;
+      const int spos = 32 * kTmodeC;
+      auto util = [&](int W, double S) {   // busy fraction of a W-warp team on an S-strip pair
+        return std::min(1.0, qsteps / (W * lag)) * S / (W * std::ceil(S / W));
+      };
+      auto item_time = [&](int W, double S) {
+        return std::max(std::ceil(S / W) * qsteps, (S - 1.0) * lag + qsteps);
+      };
+      const int kBig = 16;
+      double best_est = 1e300;
+      int bestW = 1, best_big = 1 << 30;
+      // (single-warp teams measured slower than the model says: not considered)
+      for (int W = std::min(2, t_warps); W <= t_warps; W *= 2) {
+        if (t_warps % W) continue;
+        for (int phase1 = 0; phase1 < 2; ++phase1) {
+          if (phase1 && W == t_warps) continue;
+          double t_steps = 0.0, tail = 0.0;
+          for (int pp = 0; pp < n_long; ++pp) {
+            const double S = std::ceil((double)h->db->h_pair_ncols[pp] / spos);
+            const int Wi = (phase1 && S >= kBig) ? t_warps : W;
+            t_steps += S * qsteps / util(Wi, S);
+            tail = std::max(tail, item_time(Wi, S));
+          }
+          const double est = std::max(t_steps / nw, tail) * (phase1 ? 1.05 : 1.0);
+          if (est < best_est) { best_est = est; bestW = W; best_big = phase1 ? kBig : (1 << 30); }
+        }
+      }
+      int W = bestW;
+      if (const char* f = getenv("SW_T_TEAM")) W = std::max(1, std::min(t_warps, atoi(f)));
+      while (t_warps % W) --W;
+      t.team_warps = W;
+      t.big_strips = best_big;
+      if (const char* f = getenv("SW_T_BIG")) t.big_strips = std::max(1, atoi(f));
+    }
     t.rb = s.d_rb_t;
     t.rb_cols = qcols + kPadCols + 1;
     SW_CUDA(h, launch_tmode(t, t_grid, t_smem, s.aux));

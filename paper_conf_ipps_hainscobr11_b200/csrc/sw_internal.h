@@ -101,6 +101,7 @@ KernelConfig recompute_config();
 // per lane, one CTA team of up to kTmodeThreads / 32 warps per long pair.
 constexpr int kTmodeC = 16;
 constexpr int kTmodeThreads = 256;
+constexpr int kTmodeMaxQuery = 3072;     // longer queries take team mode for long pairs
 struct TParams {
   const int8_t* matrix;      // A x A, [query][db]
   int A, rho, sigma, max_w, pad_letter;
