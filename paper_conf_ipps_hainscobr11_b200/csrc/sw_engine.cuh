@@ -416,9 +416,22 @@ __device__ __forceinline__ void emit(const SearchParams& p, uint32_t b, int pair
 // fetches it for the next strip at step T + len + 4 + j >= T + 52 + j (__syncwarp every group
 // in between).  A pair's score is reduced across the lanes once its last lane has moved on
 // (each lane parks its maximum in bdone when it leaves the pair's last strip).
+// Warp-uniform scheduler state of group_stream, kept in shared memory (one per warp): it is
+// touched once per 4-step group, and keeping it out of registers leaves the register file to
+// the R-row DP state (e[R], u[R], profile words): no spills at R = 43 with 3 warps per
+// scheduler.  Every lane executes the same updates (same addresses and values).
+struct GsState {
+  int64_t f_off;    // column offset of the pair being fetched (u16 units)
+  int64_t nx_off;   // prefetched next pair's column offset
+  int f_pair, f_len, f_P, f_col, f_seg, fn;
+  int nx_pair, nx_len;
+  int pending, e_pair, e_due;
+  uint32_t desc[2];
+};
+
 template <class L, int R>
 __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainConst& c, const uint8_t* pbase,
-                                             uint2* __restrict__ rb) {
+                                             uint2* __restrict__ rb, volatile GsState* gs) {
   static_assert(R % 4 == 0 || R >= 12, "R < 12 must be a multiple of 4");
   constexpr int kGap = 4;
   const int lane = threadIdx.x & 31;
@@ -428,54 +441,52 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
   constexpr int kStripBytes = chunks_per_lane<R>() * 32 * CB;   // chunks x 32 lanes x CB bytes
   constexpr int kEndLen = 0xffffff;            // the END segment (after the last pair) never ends
   const int passes = p.short_passes;
-  const int nshort = p.n_pairs - p.short_begin;
   const int ls = p.lg.ls;
 
   // ---- warp-uniform fetch cursor: lane 0's stream, one group (4 positions) ahead of lane 0
-  auto take = [&]() -> int {
-    int b = 0;
-    if (lane == 0) b = atomicAdd(&p.work[1], 1);
-    return __shfl_sync(SWB_FULL, b, 0);
-  };
-  int nx_pair = -1, nx_len = kEndLen;
-  int64_t nx_off = 0;
   auto prefetch = [&]() {   // next pair of the queue (its header loads overlap the current pair)
-    const int item = take();
-    if (item < nshort) {
-      nx_pair = p.short_begin + item;
-      nx_off = p.pair_off[nx_pair];
-      nx_len = p.pair_ncols[nx_pair] + kGap;
+    int item = 0;
+    if (lane == 0) item = atomicAdd(&p.work[1], 1);
+    item = __shfl_sync(SWB_FULL, item, 0);
+    if (item < p.n_pairs - p.short_begin) {
+      const int pr = p.short_begin + item;
+      gs->nx_pair = pr;
+      gs->nx_off = p.pair_off[pr];
+      gs->nx_len = p.pair_ncols[pr] + kGap;
     } else {
-      nx_pair = -1; nx_len = kEndLen;
+      gs->nx_pair = -1; gs->nx_len = kEndLen;
     }
+    __syncwarp();
   };
   prefetch();
-  if (nx_pair < 0) return;
-  int f_pair = nx_pair, f_len = nx_len, f_P = 0, f_col = 0;
-  const uint16_t* f_cols = p.cols + nx_off;
-  const uint16_t* f_pad = f_cols + (f_len - kGap);   // the pair's trailing pad columns
-  nx_pair = -2;                                   // -2: the next pair is not fetched yet
-  if (passes == 1) prefetch();
+  if (gs->nx_pair < 0) return;
+  gs->f_pair = gs->nx_pair; gs->f_len = gs->nx_len; gs->f_P = 0; gs->f_col = 0;
+  gs->f_off = gs->nx_off;
   // descriptors (len | (P + 1) << 24) of the two newest segments, by segment parity
-  uint32_t desc0 = (uint32_t)f_len | (1u << 24), desc1 = 0;
-  int f_seg = 0;
-  int fn = 0;                 // index of the next fetch (= the step at which lane 0 consumes it)
-  bool pending = false;       // a finished pair waits for its cross-lane reduction
-  int e_pair = 0, e_due = 0;
+  gs->desc[0] = (uint32_t)gs->f_len | (1u << 24); gs->desc[1] = 0;
+  gs->f_seg = 0;
+  gs->fn = 0;                 // index of the next fetch (= the step at which lane 0 consumes it)
+  gs->pending = 0;            // a finished pair waits for its cross-lane reduction
+  gs->e_pair = 0; gs->e_due = 0;
+  gs->nx_pair = -2;           // -2: the next pair is not fetched yet
+  __syncwarp();
+  if (passes == 1) prefetch();
   // this group's 4 fetches: residues g_cols[k] and top-boundary rows g_rb[k]
   const uint16_t* g_cols;
   const uint2* g_rb;
   auto plan_group = [&]() {   // warp-uniform
+    int f_pair = gs->f_pair, f_len = gs->f_len, f_P = gs->f_P, f_col = gs->f_col;
     if (f_col == f_len) {     // the next segment starts: this group fetches its gap
       if (f_P + 1 < passes) {
         ++f_P;
       } else {
-        pending = true; e_pair = f_pair; e_due = fn + 35;
-        if (nx_pair == -2) prefetch();
-        if (nx_pair >= 0) {
-          f_pair = nx_pair; f_len = nx_len; f_cols = p.cols + nx_off; f_P = 0;
-          f_pad = f_cols + (f_len - kGap);
-          nx_pair = -2;
+        gs->pending = 1; gs->e_pair = f_pair; gs->e_due = gs->fn + 35;
+        __syncwarp();
+        if (gs->nx_pair == -2) prefetch();
+        if (gs->nx_pair >= 0) {
+          f_pair = gs->nx_pair; f_len = gs->nx_len; gs->f_off = gs->nx_off; f_P = 0;
+          gs->nx_pair = -2;
+          __syncwarp();
           if (passes == 1) prefetch();
         } else {
           f_pair = -1; f_len = kEndLen; f_P = -1;   // END: gap positions for ever
@@ -483,22 +494,26 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
       }
       if (f_pair >= 0 && f_P == passes - 1 && passes > 1) prefetch();
       f_col = 0;
-      ++f_seg;
-      const uint32_t d = (uint32_t)f_len | ((uint32_t)(f_P + 1) << 24);
-      if (f_seg & 1) desc1 = d; else desc0 = d;
+      const int f_seg = gs->f_seg + 1;
+      gs->f_seg = f_seg;
+      gs->desc[f_seg & 1] = (uint32_t)f_len | ((uint32_t)(f_P + 1) << 24);
+      gs->f_pair = f_pair; gs->f_len = f_len; gs->f_P = f_P;
     }
     // residues one position ahead (look-ahead u, cell_rows): position f_col + k reads the
     // letters of column f_col + k - kGap + 1; in the gap that is the pad column(s) stored just
-    // before the pair (kLeadCols / the previous pair's trailing pads), then its first column
-    if (f_pair < 0) {                   // END: pad letters (the last pair's trailing pad columns)
-      g_cols = f_pad;
+    // before the pair (kLeadCols / the previous pair's trailing pads), then its first column.
+    // END: pad letters (the last pair's trailing pad columns, still at f_off + f_len).
+    const uint16_t* f_cols = p.cols + gs->f_off;
+    if (f_pair < 0) {
+      g_cols = f_cols + p.pair_ncols[gs->e_pair];
       g_rb = p.rb_zero;
     } else {
       g_cols = f_cols + (f_col - kGap + 1);
       g_rb = (f_col >= kGap && f_P > 0) ? rb + (f_col - kGap) : p.rb_zero;
     }
-    if (f_pair >= 0) f_col += 4;
-    fn += 4;
+    if (f_pair >= 0) gs->f_col = f_col + 4;
+    gs->fn = gs->fn + 4;
+    __syncwarp();
   };
   uint32_t ring_res[4], ring_h[4], ring_f[4];
   auto fetch = [&](int k) {
@@ -535,7 +550,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
     cell_rows<L, R>(e, u, wlo, whi, nrho, nsig, hup, fs, best);
     y_hr = hup; y_f = fs; y_res = x_res;
     // keep the next step's residue shuffle (and so its profile loads) after this step's rows:
-    // hoisting them would keep a second set of profile words live (register spills at R = 44)
+    // hoisting them would keep a second set of profile words live
     asm volatile("" : "+r"(y_res) : "r"(fs));
     if (store_rb) {
       const int pos = my_pos + K;
@@ -548,7 +563,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
     if (my_pos >= my_len) {
       if (my_pos > my_len) { y_hr = 0u; y_f = 0u; }   // last step was a stale gap cell
       ++my_seg;
-      const uint32_t d = (my_seg & 1) ? desc1 : desc0;
+      const uint32_t d = gs->desc[my_seg & 1];
       if (my_P == passes - 1) { bdone = best; best = 0; }
       my_pos -= my_len;
       my_len = (int)(d & (uint32_t)kEndLen);
@@ -559,14 +574,15 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
       for (int r = 0; r < R; ++r) { e[r] = nrho; u[r] = 0u; }
     }
     __syncwarp();
-    if (pending && S >= e_due) {   // every lane has parked the finished pair's maximum
+    if (gs->pending && S >= gs->e_due) {   // every lane has parked the finished pair's maximum
       uint32_t b = bdone;
 #pragma unroll
       for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
-      if (lane == 0) emit<L>(p, b, e_pair, 0);
-      pending = false;
+      if (lane == 0) emit<L>(p, b, gs->e_pair, 0);
+      __syncwarp();
+      gs->pending = 0;
     }
-    if (f_pair < 0 && !pending) break;
+    if (gs->f_pair < 0 && !gs->pending) break;
     plan_group();   // the 4 fetches issued during this group (consumed in the next one)
     step(std::integral_constant<int, 0>{});
     step(std::integral_constant<int, 1>{});
@@ -668,8 +684,9 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
   if constexpr (G == 32) {
     if (p.item_list == nullptr && p.group_stream) {
       constexpr int CBs = chunk_bytes<Rs>();
+      __shared__ GsState sgs[kWarps];
       group_stream<L, Rs>(p, c, smem + p.lg.off + lane * CBs,
-                              p.rb_group + (int64_t)(blockIdx.x * kWarps + warp) * p.rb_group_cols);
+                          p.rb_group + (int64_t)(blockIdx.x * kWarps + warp) * p.rb_group_cols, &sgs[warp]);
       return;
     }
   }
