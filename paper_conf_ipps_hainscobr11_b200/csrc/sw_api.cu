@@ -452,7 +452,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   const int G = pl.cfg.G;
   size_t rbg = 0;
   if (pl.short_passes > 1 && max_cols_short > 0)
-    rbg = (size_t)pl.grid * (pl.cfg.threads / 32) * (32 / G) * max_cols_short * sizeof(uint2);
+    rbg = (size_t)pl.grid * (pl.cfg.threads / 32) * (32 / G) * (max_cols_short + 4) * sizeof(uint2);
   size_t rbt = 0;
   if (pl.long_passes > 1 && n_long > 0 && !use_t) {
     const int nteams = (pl.cfg.threads / 32) / pl.team_warps;
@@ -516,13 +516,14 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   p.item_count = nullptr;
   p.work = s.d_work;
   p.rb_zero = reinterpret_cast<const uint2*>(s.d_work + 4);
+  p.hi_mul = 1u << 24;
   p.ovf_list = s.d_ovf_list;
   p.ovf_count = s.d_ovf_count;
   p.short_passes = pl.short_passes;
   p.long_passes = pl.long_passes;
   p.team_warps = pl.team_warps;
   p.rb_group = s.d_rb_group;
-  p.rb_group_cols = max_cols_short;
+  p.rb_group_cols = max_cols_short + 4;   // + 4 leading entries (group_stream gap-position stores)
   // (the stream addresses columns with 32-bit indices)
   p.group_stream = group_stream_enabled() && h->db->h_pair_off[h->db->n_pairs] < (int64_t)INT32_MAX;
   p.rb_team = s.d_rb_team;
@@ -599,6 +600,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
     }
     t.rb = s.d_rb_t;
     t.rb_cols = qcols + kPadCols + 1;
+    t.hi_mul = 1u << 24;
     SW_CUDA(h, launch_tmode(t, t_grid, t_smem, s.aux));
     SW_CUDA(h, cudaEventRecord(s.join, s.aux));
   }

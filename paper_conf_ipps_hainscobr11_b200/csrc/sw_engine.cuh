@@ -212,6 +212,7 @@ __device__ __forceinline__ uint32_t pass_tag(int pass, int cols_done) {
 struct ChainConst {
   int rho, sigma;
   uint32_t padpair;       // residue pair of two pad letters
+  uint32_t hi_mul;        // 1 << 24 at run time (SearchParams::hi_mul)
 };
 
 // The cell update (one row r of one column j, both sequences of the pair), in the
@@ -328,13 +329,15 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
     if (gl == 0) { x_hr = rh[K]; x_f = rf[K]; x_res = rr[K]; }
     // query-profile words for the two letters of the NEXT column (look-ahead u)
     uint32_t wlo[(R + 3) / 4], whi[(R + 3) / 4];
-    {
+    if constexpr (L::kSeqs == 2) {
+      // letter offsets with FMA-pipe ops only: a_hi = x >> 8 as IMAD.HI, a_lo = x - 256 a_hi
+      const int ahi = (int)__umulhi(x_res, c.hi_mul);
+      const int off_hi = ahi * ls;
+      load_prof<R, CB, GC * CB>(wlo, prow + ((int)x_res * ls - off_hi * 256));
+      load_prof<R, CB, GC * CB>(whi, prow + hi_off + off_hi);
+    } else {
       const int alo = (x_res >> hshift) & 0xff;
       load_prof<R, CB, GC * CB>(wlo, prow + alo * ls);
-      if constexpr (L::kSeqs == 2) {
-        const int ahi = x_res >> 8;
-        load_prof<R, CB, GC * CB>(whi, prow + hi_off + ahi * ls);
-      }
     }
     uint32_t hup = x_hr, fs = x_f;
     cell_rows<L, R>(e, u, wlo, whi, nrho, nsig, hup, fs, best);
@@ -441,7 +444,8 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
   constexpr int kStripBytes = chunks_per_lane<R>() * 32 * CB;   // chunks x 32 lanes x CB bytes
   constexpr int kEndLen = 0xffffff;            // the END segment (after the last pair) never ends
   const int passes = p.short_passes;
-  const int ls = p.lg.ls;
+  const int ls = p.lg.ls, ls256 = ls * 256;
+  const uint32_t hi_mul = p.hi_mul;
 
   // ---- warp-uniform fetch cursor: lane 0's stream, one group (4 positions) ahead of lane 0
   auto prefetch = [&]() {   // next pair of the queue (its header loads overlap the current pair)
@@ -543,8 +547,14 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
     uint32_t x_res = __shfl_up_sync(SWB_FULL, y_res, 1);
     if (lane == 0) { x_hr = ring_h[K]; x_f = ring_f[K]; x_res = ring_res[K]; }
     uint32_t wlo[(R + 3) / 4], whi[(R + 3) / 4];   // profile words of the next position's letters
-    load_prof<R, CB, 32 * CB>(wlo, prow + (x_res & 0xff) * ls);
-    load_prof<R, CB, 32 * CB>(whi, prow + (x_res >> 8) * ls);
+    {
+      // letter offsets with FMA-pipe ops only: a_hi = x >> 8 as IMAD.HI, a_lo = x - 256 a_hi
+      const int ahi = (int)__umulhi(x_res, hi_mul);
+      const int off_hi = ahi * ls;
+      const int off_lo = (int)x_res * ls - ahi * ls256;
+      load_prof<R, CB, 32 * CB>(wlo, prow + off_lo);
+      load_prof<R, CB, 32 * CB>(whi, prow + off_hi);
+    }
     fetch(K);
     uint32_t hup = x_hr, fs = x_f;
     cell_rows<L, R>(e, u, wlo, whi, nrho, nsig, hup, fs, best);
@@ -552,10 +562,9 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
     // keep the next step's residue shuffle (and so its profile loads) after this step's rows:
     // hoisting them would keep a second set of profile words live
     asm volatile("" : "+r"(y_res) : "r"(fs));
-    if (store_rb) {
-      const int pos = my_pos + K;
-      if (pos >= kGap && pos < my_len) rb[pos - kGap] = make_uint2(hup, fs);
-    }
+    // unconditional for the storing lane: gap positions land in the slot's kGap leading
+    // entries, stale positions past the segment beyond its columns; neither is ever read
+    if (store_rb) rb[my_pos + K - kGap] = make_uint2(hup, fs);
   };
 
   for (int S = 0;; S += 4) {
@@ -625,6 +634,7 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
   c.rho = p.rho;
   c.sigma = p.sigma;
   c.padpair = (uint32_t)p.pad_letter | ((uint32_t)p.pad_letter << 8);
+  c.hi_mul = p.hi_mul;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
@@ -686,7 +696,7 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
       constexpr int CBs = chunk_bytes<Rs>();
       __shared__ GsState sgs[kWarps];
       group_stream<L, Rs>(p, c, smem + p.lg.off + lane * CBs,
-                          p.rb_group + (int64_t)(blockIdx.x * kWarps + warp) * p.rb_group_cols, &sgs[warp]);
+                          p.rb_group + (int64_t)(blockIdx.x * kWarps + warp) * p.rb_group_cols + 4, &sgs[warp]);
       return;
     }
   }
@@ -844,6 +854,7 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   c.rho = p.rho;
   c.sigma = p.sigma;
   c.padpair = (uint32_t)p.pad_letter | ((uint32_t)p.pad_letter << 8);
+  c.hi_mul = p.hi_mul;
   uint8_t* tab = tables + warp * table_bytes;
   uint2* rb_cta = p.rb + (int64_t)blockIdx.x * (2 * p.warps) * p.rb_cols;
   // Phase 1: one team of all warps for the longest pairs (items come longest-first), so the

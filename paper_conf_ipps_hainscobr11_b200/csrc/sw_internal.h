@@ -74,6 +74,8 @@ struct SearchParams {
   uint2* rb_group; int64_t rb_group_cols;   // per group slot (>= max n' + kPadCols)
   int group_stream;          // G = 32: continuous stream over strips and pairs (group_stream)
   const uint2* rb_zero;      // 4 neutral row-buffer entries (H = 0, F + rho = 0)
+  uint32_t hi_mul;           // 1 << 24, as a runtime value: umulhi(pair, hi_mul) = pair >> 8 on
+                             // the FMA pipe (IMAD.HI), keeping letter extraction off the ALU pipe
   uint2* rb_team;  int64_t rb_team_cols;    // per (team slot, pass mod (team_warps+1))
 };
 
@@ -121,6 +123,7 @@ struct TParams {
   int team_warps;            // warps per team in phase 2 (divides warps)
   int big_strips;            // phase 1 (one team of all warps) keeps pairs with >= big_strips strips
   uint2* rb; int64_t rb_cols;   // per CTA: 2 * warps slots (teams x (team_warps + 1) <= 2 * warps)
+  uint32_t hi_mul;           // 1 << 24 (see SearchParams::hi_mul)
 };
 
 cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st);
