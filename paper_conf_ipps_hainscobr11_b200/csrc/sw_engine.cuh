@@ -215,37 +215,46 @@ struct ChainConst {
   uint32_t hi_mul;        // 1 << 24 at run time (SearchParams::hi_mul)
 };
 
-// The cell update (one row r of one column j, both sequences of the pair), in the
-// "look-ahead" form used by every mode: besides E, each row keeps u = max(H[r-1][j] + w(q_r,
-// d_{j+1}), E[r][j+1], 0) for the NEXT column, formed as soon as its inputs exist (the row
-// above's H at this column and this row's new E).  Then every per-row register (e[r], u[r]) is
-// read and rewritten by its own row only, so the unrolled step loop needs no register
-// rotation (the previous form kept H - rho of the left column per row, whose old value had to
-// survive one row longer than its new one: ~R register moves per step, or 2R registers).
-//   fs   = max(fs - sigma, h_up)          F + rho of this row      VIADDMNMX
-//   h    = max(fs - rho, u[r])            H[r][j]                  VIADDMNMX
+// The cell update (one row r of one column j, both sequences of the pair).  Besides E, each row
+// keeps t = H[r-1][j] + w(q_r, d_{j+1}) for the NEXT column (the diagonal term of Eq.(1)),
+// formed as soon as its inputs exist (the row above's H at this column).  Every per-row
+// register (e[r], t[r]) is read and rewritten by its own row only, so the unrolled step loop
+// needs no register rotation (an earlier form kept H - rho of the left column per row, whose
+// old value had to survive one row longer than its new one: ~R register moves per step).
+//   f    = max(f - sigma, hr_up)          F[r][j]                  VIADDMNMX
+//   h    = max(t[r], e[r], f, 0)          H[r][j]                  VIMNMX3.RELU
 //   hr   = h - rho                                                 VIADD.16x2 (FMA pipe)
 //   e[r] = max(e[r] - sigma, hr)          E[r][j+1]                VIADDMNMX
-//   u[r] = max(hr_up + (w + rho), e[r], 0)  for column j+1         VIADDMNMX.RELU
+//   t[r] = hr_up + (w + rho)              for column j+1           VIADD.16x2 (FMA pipe)
 //   best = max(best, h, h') every two rows                         VIMNMX3
-// plus one PRMT per row for w + rho of column j+1 (profile words of the next column's letters).
+// plus one PRMT per row for w + rho of column j+1 (profile words of the next column's letters):
+// 4.5 ALU-pipe + 2 FMA-pipe instructions per cell pair.  (The earlier "u" form,
+// u = max(T, E, 0) by VIADDMNMX.RELU and H = max(F + rho - rho, u) by VIADDMNMX, kept the
+// vertical chain at two ALU ops but spent 5.5 ALU-pipe instructions per cell pair; here the
+// 3-input max with the zero clamp takes T, E and F at once and the adds move to the FMA pipe.
+// The chain f -> h -> hr -> f now runs through the FMA pipe (~13 cycles per row); forming
+// F - sigma beside H to keep it at two ALU ops cost one more FMA-pipe instruction per cell
+// pair and measured 4-5 % slower: issue slots, not the chain, are the tighter limit.)
+// Vertical values enter and leave as (H, F + rho), the format of the lane hand-off and of the
+// strip row buffers.
 template <class L, int R>
-__device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&u)[R], const uint32_t (&wlo)[(R + 3) / 4],
-                                          const uint32_t (&whi)[(R + 3) / 4], uint32_t nrho, uint32_t nsig,
-                                          uint32_t& hup, uint32_t& fs, uint32_t& best) {
-  uint32_t hrup = L::add(hup, nrho), hprev = 0;
+__device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&t)[R], const uint32_t (&wlo)[(R + 3) / 4],
+                                          const uint32_t (&whi)[(R + 3) / 4], uint32_t nrho, uint32_t prho,
+                                          uint32_t nsig, uint32_t& hup, uint32_t& fs, uint32_t& best) {
+  uint32_t hrup = L::add(hup, nrho), f = L::add(fs, nrho), hprev = 0, h = 0;
 #pragma unroll
   for (int r = 0; r < R; ++r) {
-    fs = L::gap(fs, nsig, hup);                                       // F + rho = max(F[i-1] + rho - sigma, H[i-1])
-    const uint32_t h = L::gap(fs, nrho, u[r]);                        // H = max(F, u)
+    f = L::gap(f, nsig, hrup);                                        // F = max(F[i-1] - sigma, H[i-1] - rho)
+    h = L::hmax(t[r], e[r], f);                                       // H = max(H[i-1][j-1] + w, E, F, 0)
     const uint32_t hr = L::add(h, nrho);                              // H - rho
     e[r] = L::gap(e[r], nsig, hr);                                    // E[j+1] = max(E - sigma, H - rho)
-    u[r] = L::hcell(hrup, subst_row<L, R>(wlo, whi, r), e[r]);        // max(H[i-1][j] + w(q_i, d_{j+1}), E[j+1], 0)
+    t[r] = L::add(hrup, subst_row<L, R>(wlo, whi, r));                // H[i-1][j] + w(q_i, d_{j+1})
     hrup = hr;
-    hup = h;
     if (r & 1) best = L::max3(best, hprev, h); else hprev = h;
   }
   if constexpr (R & 1) best = L::max2(best, hprev);
+  hup = h;
+  fs = L::add(f, prho);                                               // F + rho for the lane below
 }
 
 // One strip pass of a chain of GC lanes over the columns of one database pair (see the file
@@ -267,16 +276,16 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
   static_assert(R % 4 == 0 || R >= 12, "R < 12 must be a multiple of 4");
   const int lane = threadIdx.x & 31;
   const int gl = lane & (GC - 1);
-  const uint32_t nrho = L::splat(-c.rho);
+  const uint32_t nrho = L::splat(-c.rho), prho = L::splat(c.rho);
   const uint32_t nsig = L::splat(-c.sigma);
   const int hshift = 8 * half;
   constexpr int CB = chunk_bytes<R>();
   const bool store_out = (gl == GC - 1) && (P < passes_total - 1);
   const bool from_prev = P > 0;
 
-  uint32_t e[R], u[R];
+  uint32_t e[R], t[R];
 #pragma unroll
-  for (int r = 0; r < R; ++r) { e[r] = nrho; u[r] = 0u; }
+  for (int r = 0; r < R; ++r) { e[r] = nrho; t[r] = 0u; }
   uint32_t y_hr = 0, y_f = 0, y_res = c.padpair;   // (H, F + rho) of this lane's bottom row
   int col = -gl - 1;
 
@@ -340,7 +349,7 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
       load_prof<R, CB, GC * CB>(wlo, prow + alo * ls);
     }
     uint32_t hup = x_hr, fs = x_f;
-    cell_rows<L, R>(e, u, wlo, whi, nrho, nsig, hup, fs, best);
+    cell_rows<L, R>(e, t, wlo, whi, nrho, prho, nsig, hup, fs, best);
     y_hr = hup; y_f = fs; y_res = x_res;
     // last lane: save the strip's bottom row for the next strip (not after the last strip);
     // fill steps write neutral values (index -1 keeps its neutral entry) that the real column
@@ -438,7 +447,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
   static_assert(R % 4 == 0 || R >= 12, "R < 12 must be a multiple of 4");
   constexpr int kGap = 4;
   const int lane = threadIdx.x & 31;
-  const uint32_t nrho = L::splat(-c.rho);
+  const uint32_t nrho = L::splat(-c.rho), prho = L::splat(c.rho);
   const uint32_t nsig = L::splat(-c.sigma);
   constexpr int CB = chunk_bytes<R>();
   constexpr int kStripBytes = chunks_per_lane<R>() * 32 * CB;   // chunks x 32 lanes x CB bytes
@@ -527,9 +536,9 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
   };
 
   // ---- per-lane state (look-ahead form, cell_rows)
-  uint32_t e[R], u[R];
+  uint32_t e[R], t[R];
 #pragma unroll
-  for (int r = 0; r < R; ++r) { e[r] = nrho; u[r] = 0u; }
+  for (int r = 0; r < R; ++r) { e[r] = nrho; t[r] = 0u; }
   uint32_t y_hr = 0, y_f = 0, y_res = c.padpair;
   uint32_t best = 0, bdone = 0;
   int my_pos = -lane, my_len = 0, my_P = -1, my_seg = -1;   // lane l reaches segment 0 at step l
@@ -557,7 +566,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
     }
     fetch(K);
     uint32_t hup = x_hr, fs = x_f;
-    cell_rows<L, R>(e, u, wlo, whi, nrho, nsig, hup, fs, best);
+    cell_rows<L, R>(e, t, wlo, whi, nrho, prho, nsig, hup, fs, best);
     y_hr = hup; y_f = fs; y_res = x_res;
     // keep the next step's residue shuffle (and so its profile loads) after this step's rows:
     // hoisting them would keep a second set of profile words live
@@ -580,7 +589,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
       store_rb = lane == 31 && my_P >= 0 && my_P < passes - 1;
       prow = pbase + max(my_P, 0) * kStripBytes;
 #pragma unroll
-      for (int r = 0; r < R; ++r) { e[r] = nrho; u[r] = 0u; }
+      for (int r = 0; r < R; ++r) { e[r] = nrho; t[r] = 0u; }
     }
     __syncwarp();
     if (gs->pending && S >= gs->e_due) {   // every lane has parked the finished pair's maximum

@@ -112,11 +112,11 @@ constexpr int CM_R = 32;
 constexpr int CM_COLS = 256;
 __global__ void __launch_bounds__(512) k_cellmix(uint32_t* out, uint32_t seed, Rec* rec) {
   constexpr int R = CM_R;
-  uint32_t hr[R], e[R];
-  const uint32_t nsig = 0xFFFEFFFEu, nrho = 0xFFF6FFF6u;
+  uint32_t t[R], e[R];
+  const uint32_t nsig = 0xFFFEFFFEu, nrho = 0xFFF6FFF6u, prho = 0x000A000Au;
 #pragma unroll
-  for (int r = 0; r < R; ++r) { hr[r] = nrho; e[r] = nrho; }
-  uint32_t best = 0, hup0 = 0, fs0 = 0, hrdiag0 = nrho;
+  for (int r = 0; r < R; ++r) { t[r] = 0u; e[r] = nrho; }
+  uint32_t best = 0, hup0 = 0, fs0 = 0;
   // profile: 16 letters x R rows of int8, per-lane copy so the LDS.128 are conflict-free
   __shared__ __align__(16) uint8_t sprof[16 * R * 32];
   for (int i = threadIdx.x; i < 16 * R * 32; i += blockDim.x) sprof[i] = (uint8_t)((seed + i * 37u) % 23u);
@@ -138,7 +138,9 @@ __global__ void __launch_bounds__(512) k_cellmix(uint32_t* out, uint32_t seed, R
       wlo[4 * k] = a.x; wlo[4 * k + 1] = a.y; wlo[4 * k + 2] = a.z; wlo[4 * k + 3] = a.w;
       whi[4 * k] = bb.x; whi[4 * k + 1] = bb.y; whi[4 * k + 2] = bb.z; whi[4 * k + 3] = bb.w;
     }
-    uint32_t hup = hup0, fs = fs0, hrdiag = hrdiag0, hprev = 0;
+    // the engine's cell update (sw_engine.cuh cell_rows): F, H = max3.relu(T, E, F), H - rho,
+    // E, T of the next column, best every two rows
+    uint32_t hrup = __vadd2(hup0, nrho), f = __vadd2(fs0, nrho), hprev = 0, h = 0;
 #pragma unroll
     for (int r = 0; r < R; ++r) {
       uint32_t w;
@@ -148,25 +150,23 @@ __global__ void __launch_bounds__(512) k_cellmix(uint32_t* out, uint32_t seed, R
         case 2: w = prmt_imm<0xE6A2u>(wlo[r >> 2], whi[r >> 2]); break;
         default: w = prmt_imm<0xF7B3u>(wlo[r >> 2], whi[r >> 2]); break;
       }
-      e[r] = __viaddmax_s16x2(e[r], nsig, hr[r]);
-      const uint32_t u = __viaddmax_s16x2_relu(hrdiag, w, e[r]);
-      fs = __viaddmax_s16x2(fs, nsig, hup);
-      const uint32_t h = __viaddmax_s16x2(fs, nrho, u);
-      hrdiag = hr[r];
-      hr[r] = __vadd2(h, nrho);
-      hup = h;
+      f = __viaddmax_s16x2(f, nsig, hrup);
+      h = __vimax3_s16x2_relu(t[r], e[r], f);
+      const uint32_t hr = __vadd2(h, nrho);
+      e[r] = __viaddmax_s16x2(e[r], nsig, hr);
+      t[r] = __vadd2(hrup, w);
+      hrup = hr;
       if (r & 1) best = __vimax3_s16x2(best, hprev, h); else hprev = h;
     }
     // the next column's top input: this lane's bottom row (a chain of one lane)
-    hrdiag0 = __vadd2(hup0, nrho);
-    hup0 = hup; fs0 = fs;
+    hup0 = h; fs0 = __vadd2(f, prho);
   }
   __syncthreads();
   long long t1 = clock64();
   unsigned long long g1 = gtimer();
   uint32_t acc = best;
 #pragma unroll
-  for (int r = 0; r < R; ++r) acc ^= hr[r] ^ e[r];
+  for (int r = 0; r < R; ++r) acc ^= t[r] ^ e[r];
   if (acc == 0x12345678u) out[blockIdx.x * blockDim.x + threadIdx.x] = acc;
   if (threadIdx.x == 0) rec[blockIdx.x] = Rec{t0, t1, g0, g1, smid(), 0};
 }
@@ -250,7 +250,7 @@ int main() {
   run("cellmix_cells", k_cellmix, (ITERS / 4) * CM_R * 2.0, threads, d_out, d_rec, false);
   printf(", \"cells_per_clk_per_gpu\": %.2f, \"sm_mhz_during\": %.0f, \"what\": \"rates = warp-instructions (cellmix: "
          "warp-cells) per SM clock over the per-SM window in which the blocks ran; cells_per_clk_per_gpu = 32 lanes x "
-         "SMs x the cell-mix rate (PRMT + 5 DPX + 0.5 VIMNMX3 per 2 cells, profile from smem via LDS.128)\"}\n",
+         "SMs x the cell-mix rate (per 2 cells: PRMT + 2 VIADDMNMX + VIMNMX3.RELU + 0.5 VIMNMX3 on the ALU pipe, 2 VIADD.16x2 on the FMA pipe; profile from smem via LDS.128)\"}\n",
          g_rate * 32.0 * nsm, g_clk * 1e3);
   cudaError_t err = cudaGetLastError();
   if (err != cudaSuccess) { fprintf(stderr, "CUDA error %s\n", cudaGetErrorString(err)); return 1; }
