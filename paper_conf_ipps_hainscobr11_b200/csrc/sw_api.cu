@@ -254,14 +254,16 @@ int make_plan(sw_handle h, int m, const Split& sp, Plan* pl) {
     int bytes = 0;
     main_layouts(c, m, A1, &lg, &lt, &bytes);
     if (bytes > kMaxProfileSmem) continue;
-    // several strips in group mode are only efficient for whole-warp chains: with G < 32 the
-    // strip-boundary row traffic per cell grows by 32 / G and its latency dominates (measured)
-    if (lg.strips > 1 && c.G < 32) continue;
-    // ALU instructions per step; a config with more resident warps per scheduler hides the
-    // 2 x 4.4-cycle F/H dependency chain better (measured: 3 warps ~2.5 % faster than 2)
+    // several strips with G < 32 (run_pass per strip): each strip pays its own pipeline fill
+    // (counted below) and the row-buffer store / ring fetch per step (~8 instructions);
+    // measured best for m = 464-1000 (profiles/r01_plan_check.jsonl)
+    const double strip_extra = (lg.strips > 1 && c.G < 32) ? 8.0 : 0.0;
+    // ALU instructions per step; 2 warps per scheduler hide the F -> H -> H - rho chain (~13
+    // cycles per row, through the FMA pipe) worse than 3: measured +11 % time (R = 43, 256 vs
+    // 384 threads, profiles/r01_plan_check.jsonl); 4 warps per scheduler measured no better than 3
     const double wps = c.threads / 128.0;
-    const double lat = 1.0 - 0.025 * std::min(2.0, std::max(0.0, wps - 2.0));
-    const double is = (6.5 * c.Rs + 24.0) * lat, il = (6.5 * c.Rl + 40.0) * lat;
+    const double lat = wps < 2.5 ? 1.10 : 1.0;
+    const double is = (6.5 * c.Rs + 24.0 + strip_extra) * lat, il = (6.5 * c.Rl + 40.0) * lat;
     const int W = team_warps_for(lt.strips, c.threads / 32);
     // (G = 32 streams: a 4-column gap per segment plus ~3 steps' worth of per-lane resets)
     const double fill = (c.G == 32 && group_stream_enabled()) ? 7.0 : c.G - 1.0;
@@ -286,6 +288,9 @@ int make_plan(sw_handle h, int m, const Split& sp, Plan* pl) {
   }
   if (best_i < 0) return fail(h, SW_E_UNSUPPORTED, "query profile does not fit in shared memory (query_len * (alphabet_size + 1) too large)");
   const KernelConfig c = menu_entry(best_i);
+  if (getenv("SW_DEBUG_PLAN"))
+    fprintf(stderr, "plan m=%d menu=%d G=%d Rs=%d Rl=%d threads=%d cost=%.4g\n", m, best_i, c.G, c.Rs, c.Rl, c.threads,
+            best);
   pl->cfg = c;
   main_layouts(c, m, A1, &pl->lg, &pl->lt, &pl->prof_bytes);
   if (pl->prof_bytes > kMaxProfileSmem) return fail(h, SW_E_UNSUPPORTED, "query profile does not fit in shared memory");

@@ -110,8 +110,8 @@ __device__ __forceinline__ uint32_t prmt_imm(uint32_t a, uint32_t b) {
 }
 constexpr int CM_R = 32;
 constexpr int CM_COLS = 256;
-__global__ void __launch_bounds__(512) k_cellmix(uint32_t* out, uint32_t seed, Rec* rec) {
-  constexpr int R = CM_R;
+template <int R, int NT>
+__global__ void __launch_bounds__(NT) k_cellmix(uint32_t* out, uint32_t seed, Rec* rec) {
   uint32_t t[R], e[R];
   const uint32_t nsig = 0xFFFEFFFEu, nrho = 0xFFF6FFF6u, prho = 0x000A000Au;
 #pragma unroll
@@ -247,7 +247,12 @@ int main() {
   run("VIADDMNMX+IMAD", k_peak<10, 6>, ipt, threads, d_out, d_rec, false);
   run("VIADDMNMX+IADD3", k_peak<10, 3>, ipt, threads, d_out, d_rec, false);
   // the cell mix, counted in CELLS: per column R rows x 2 cells (two sequences per s16x2 lane)
-  run("cellmix_cells", k_cellmix, (ITERS / 4) * CM_R * 2.0, threads, d_out, d_rec, false);
+  run("cellmix_cells", k_cellmix<CM_R, 512>, (ITERS / 4) * CM_R * 2.0, threads, d_out, d_rec, false);
+  const double mix_rate = g_rate;
+  // the same mix at 3 warps per scheduler (the engine's 384-thread configurations), R = 32 / 48
+  run("cellmix_cells_R32_384", k_cellmix<32, 384>, (ITERS / 4) * 32 * 2.0, 384, d_out, d_rec, false);
+  run("cellmix_cells_R48_384", k_cellmix<48, 384>, (ITERS / 4) * 48 * 2.0, 384, d_out, d_rec, false);
+  g_rate = mix_rate;
   printf(", \"cells_per_clk_per_gpu\": %.2f, \"sm_mhz_during\": %.0f, \"what\": \"rates = warp-instructions (cellmix: "
          "warp-cells) per SM clock over the per-SM window in which the blocks ran; cells_per_clk_per_gpu = 32 lanes x "
          "SMs x the cell-mix rate (per 2 cells: PRMT + 2 VIADDMNMX + VIMNMX3.RELU + 0.5 VIMNMX3 on the ALU pipe, 2 VIADD.16x2 on the FMA pipe; profile from smem via LDS.128)\"}\n",
