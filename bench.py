@@ -102,6 +102,10 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------------------- workload
+DB_DESC = {"C1": "Swiss-Prot-shaped synthetic DB (parity-small)", "C2": "Swiss-Prot-shaped synthetic DB",
+           "C4": "Swiss-Prot-shaped synthetic DB", "C3": "long-sequence synthetic DB (all > 3072 residues)"}
+
+
 def make_workload(name: str, rank: int, world: int):
     """Weak scaling: N ranks search N x (the config's database), one config-sized shard each."""
     if name in ("C2", "C4"):
@@ -204,11 +208,14 @@ def bench_ours(args, rank, world, local_rank):
 
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
-    if world > 1:
+    # the NCCL path (process group + score gather) runs for N > 1; SW_BENCH_DIST=1 also runs it
+    # at N = 1 under torchrun (a one-GPU check of the multi-GPU code path)
+    dist_on = world > 1 or os.environ.get("SW_BENCH_DIST") == "1"
+    if dist_on:
         dist.init_process_group("nccl", device_id=dev)
     if rank == 0:
         swbuild.build()
-    if world > 1:
+    if dist_on:
         dist.barrier()
     qs, db, lens_all, mat, rho, sigma, T = make_workload(args.config, rank, world)
     if args.threshold is not None:
@@ -221,7 +228,7 @@ def bench_ours(args, rank, world, local_rank):
     n_local = db.num_seqs
     n_pad = shard_size_bound(n_total, world)
     sw = swp.SmithWaterman(qs[0], W, rho, sigma)
-    if world > 1:
+    if dist_on:
         gath = ScoreGather(db.global_index, n_total, nq, device=dev)
         # shard padded with empty sequences to the uniform gather size (they score 0)
         sw.load_db(db.residues, ScoreGather.pad_offsets(db.offsets, n_pad))
@@ -245,7 +252,7 @@ def bench_ours(args, rank, world, local_rank):
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize(dev)
-    if world > 1:
+    if dist_on:
         dist.barrier()
     clocks = ClockSampler(local_rank)
     clocks.start()
@@ -255,7 +262,7 @@ def bench_ours(args, rank, world, local_rank):
     kern_ms = 0.0
     rec_ms = 0.0
     torch.cuda.synchronize(dev)
-    if world > 1:
+    if dist_on:
         dist.barrier()
     ev0.record(stream)
     for _ in range(args.steps):
@@ -271,7 +278,7 @@ def bench_ours(args, rank, world, local_rank):
     if T != -1 and not args.no_auto:
         step(-1)
         torch.cuda.synchronize(dev)
-        if world > 1:
+        if dist_on:
             dist.barrier()
         ev0.record(stream)
         for _ in range(args.steps):
@@ -279,7 +286,7 @@ def bench_ours(args, rank, world, local_rank):
         ev1.record(stream)
         torch.cuda.synchronize(dev)
         auto_ms = ev0.elapsed_time(ev1)
-        if world > 1:
+        if dist_on:
             t = torch.tensor([auto_ms], dtype=torch.float64, device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             auto_ms = float(t.item())
@@ -292,7 +299,7 @@ def bench_ours(args, rank, world, local_rank):
     os.environ.pop("SW_STREAMS", None)
     km = sw.kernel_ms()
     kern_ms, rec_ms = km["search_ms"], km["recompute_ms"]
-    if world > 1:
+    if dist_on:
         t = torch.tensor([ms], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
@@ -302,10 +309,10 @@ def bench_ours(args, rank, world, local_rank):
     t0 = time.perf_counter()
     for _ in range(e2e_steps):
         host = sw.search_batch(qs, T)
-        if world > 1:
+        if dist_on:
             dist.barrier()
     e2e_s = (time.perf_counter() - t0) / e2e_steps
-    if world > 1:
+    if dist_on:
         t = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_s = float(t.item())
@@ -321,7 +328,7 @@ def bench_ours(args, rank, world, local_rank):
         t0 = time.perf_counter()
         sw.search_stream(db.residues, db.offsets, T, chunk, queries=qs)
         st_s = time.perf_counter() - t0
-        if world > 1:
+        if dist_on:
             t = torch.tensor([st_s], dtype=torch.float64, device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             st_s = float(t.item())
@@ -334,7 +341,7 @@ def bench_ours(args, rank, world, local_rank):
 
     if rank != 0:
         sw.close()
-        if world > 1:
+        if dist_on:
             dist.destroy_process_group()
         return
     step_s = ms / 1e3 / args.steps
@@ -380,11 +387,15 @@ def bench_ours(args, rank, world, local_rank):
         "metric": "GCUPS", "value": round(gcups, 2), "unit": "GCUPS", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(1e3 * step_s, 3), "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "s16x2 (int32 recompute)", "data": "synthetic",
-        "config": {"workload": f"{args.config}: Swiss-Prot-shaped synthetic DB, 540k seqs / ~191M residues per GPU, "
+        "config": {"workload": f"{args.config}: {DB_DESC.get(args.config, 'synthetic DB')}, "
+                               f"{n_local} seqs / {db.total_residues / 1e6:.1f}M residues per GPU, "
                                f"queries {[int(q.size) for q in qs]}", "matrix": mat, "gap_open": rho,
                    "gap_extend": sigma, "threshold": T, "seqs_per_gpu": n_local,
                    "residues_per_gpu": db.total_residues, "cells_per_step": cells_total,
-                   "l2": "inputs larger than L2 (device DB ~2x191 MB > 126 MB)", "parallelism": f"db-shard x{world}"},
+                   "l2": (f"inputs larger than L2 (device DB ~{2 * db.total_residues / 1e6:.0f} MB > 126 MB)"
+                          if 2 * db.total_residues > 126e6 else
+                          f"device DB ~{2 * db.total_residues / 1e6:.0f} MB fits in L2 (small config)"),
+                   "parallelism": f"db-shard x{world}"},
         "clocks": clk,
         "e2e": {"value": round(e2e_gcups, 2), "unit": "GCUPS", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "api": "sw_search_batch (blocking, host buffers; DB resident as in PAPER.md L32)"},
@@ -401,7 +412,7 @@ def bench_ours(args, rank, world, local_rank):
     }
     print(json.dumps(line), flush=True)
     sw.close()
-    if world > 1:
+    if dist_on:
         dist.destroy_process_group()
 
 

@@ -46,6 +46,8 @@ __device__ __forceinline__ uint32_t op(uint32_t a, uint32_t b, uint32_t c) {
   if constexpr (OP == 4) asm volatile("lop3.b32 %0, %1, %2, %3, 0x96;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
   if constexpr (OP == 5) asm volatile("max.s32 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(c));
   if constexpr (OP == 6) asm volatile("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+  if constexpr (OP == 7) asm volatile("max.f16x2 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(c));
+  if constexpr (OP == 8) asm volatile("max.bf16x2 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(c));
   return d;
 }
 // DPX classes through the intrinsics (ptxas emits one SASS op each); volatile via a barrier
@@ -92,16 +94,16 @@ __global__ void __launch_bounds__(512) k_peak(uint32_t* out, uint32_t seed, Rec*
   if (threadIdx.x == 0) rec[blockIdx.x] = Rec{t0, t1, g0, g1, smid(), 0};
 }
 
-// The s16x2 Smith-Waterman cell update exactly as sw_engine.cuh's run_pass issues it, per row:
-//   e  = VIADDMNMX(e, -sigma, hr_left)
-//   u  = VIADDMNMX.RELU(hr_diag, w + rho, e)
-//   fs = VIADDMNMX(fs, -sigma, h_up)
-//   h  = VIADDMNMX(fs, -rho, u)
-//   hr = VIADD.16x2(h, -rho)
-//   w  = PRMT(profile_lo, profile_hi)          (sign-extend two int8 scores)
+// The s16x2 Smith-Waterman cell update exactly as sw_engine.cuh's cell_rows issues it, per row:
+//   f    = VIADDMNMX(f, -sigma, hr_up)
+//   h    = VIMNMX3.RELU(t, e, f)
+//   hr   = VIADD.16x2(h, -rho)                 (FMA pipe)
+//   e    = VIADDMNMX(e, -sigma, hr)
+//   t    = VIADD.16x2(hr_up, w + rho)          (FMA pipe)
+//   w    = PRMT(profile_lo, profile_hi)        (sign-extend two int8 scores)
 //   best = VIMNMX3(best, h, h') every two rows
-// = 6.5 ALU-class instructions per two cells; the profile words come from shared memory (LDS.128,
-// R/16 x 2 per column as in the engine) at a letter that changes every column.
+// = 4.5 ALU-pipe + 2 FMA-pipe instructions per two cells; the profile words come from shared
+// memory (LDS.128, R/16 x 2 per column as in the engine) at a letter that changes every column.
 template <uint32_t SEL>
 __device__ __forceinline__ uint32_t prmt_imm(uint32_t a, uint32_t b) {
   uint32_t d;
@@ -246,6 +248,9 @@ int main() {
   run("VIADDMNMX+VIADD.16x2", k_peak<10, 14>, ipt, threads, d_out, d_rec, false);
   run("VIADDMNMX+IMAD", k_peak<10, 6>, ipt, threads, d_out, d_rec, false);
   run("VIADDMNMX+IADD3", k_peak<10, 3>, ipt, threads, d_out, d_rec, false);
+  run("HMNMX2", k_peak<7, -1>, ipt, threads, d_out, d_rec, false);
+  run("VIADDMNMX+HMNMX2", k_peak<10, 7>, ipt, threads, d_out, d_rec, false);
+  run("VIADDMNMX+HMNMX2.BF16", k_peak<10, 8>, ipt, threads, d_out, d_rec, false);
   // the cell mix, counted in CELLS: per column R rows x 2 cells (two sequences per s16x2 lane)
   run("cellmix_cells", k_cellmix<CM_R, 512>, (ITERS / 4) * CM_R * 2.0, threads, d_out, d_rec, false);
   const double mix_rate = g_rate;
