@@ -7,6 +7,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <map>
 #include <numeric>
 #include <string>
 #include <thread>
@@ -111,6 +112,10 @@ struct sw_handle_s {
   uint8_t* d_tb_query = nullptr; size_t tb_query_cap = 0;
   KernelConfig last_cfg{};
   int32_t last_threshold = 0;
+  // measured plan choice per (query length, threshold) on the loaded database (run_batch
+  // autotune; -1 = keep the model's choice); cleared by sw_load_db
+  std::map<std::pair<int, int32_t>, int> tuned;
+  int tune_force = -1;            // menu entry forced while tuning / from the tuned table
   // scratch
   std::vector<QuerySlot> slots;
   int32_t* d_scores_tmp = nullptr;
@@ -241,7 +246,8 @@ struct Split {
 //    steps = sum over long pairs of (n' + 31) x strips), and
 //  * the critical path of the longest item (long: its strips split over the team's warps;
 //    short: one group), at the issue rate one warp gets while sharing its scheduler.
-int make_plan(sw_handle h, int m, const Split& sp, Plan* pl) {
+int make_plan(sw_handle h, int m, const Split& sp, Plan* pl, int force = -1,
+              std::vector<std::pair<double, int>>* ranked = nullptr) {
   const int A1 = h->A + 1;
   const double kGpuIssue = 2.7 * h->num_sms;  // ALU warp-instructions per clock, whole GPU
   const double kWarpIssue = 0.2;              // one warp's share of its scheduler
@@ -269,7 +275,11 @@ int make_plan(sw_handle h, int m, const Split& sp, Plan* pl) {
     const double fill = (c.G == 32 && group_stream_enabled()) ? 7.0 : c.G - 1.0;
     const double gsteps = ((double)sp.short_cols + (double)sp.n_short * fill) * lg.strips / (32 / c.G);
     const double tsteps = ((double)sp.long_cols + 31.0 * sp.n_long) * lt.strips;
-    double thr = (gsteps * is + tsteps * il) / kGpuIssue;
+    // team mode: a CTA holds floor(warps / W) teams; warps beyond the last whole team idle
+    // (W = 7 of 12 warps measured 32 % slower than W = 6 on C3 with query 5478)
+    const int cta_warps = c.threads / 32;
+    const double team_util = (double)((cta_warps / W) * W) / cta_warps;
+    double thr = (gsteps * is + tsteps * il / team_util) / kGpuIssue;
     // few items: the issue rate needs ~2 busy warps per scheduler (4 per SM)
     const double active_warps = (double)sp.n_short / (32 / c.G) + (double)sp.n_long * W;
     const double thr_full = thr;
@@ -277,8 +287,10 @@ int make_plan(sw_handle h, int m, const Split& sp, Plan* pl) {
     const double tail_l = sp.n_long ? (sp.long_max_cols + 31.0) * ((lt.strips + W - 1) / W) * il / kWarpIssue : 0.0;
     const double tail_s = sp.n_short ? (sp.short_max_cols + c.G - 1.0) * lg.strips * is / kWarpIssue : 0.0;
     const double cost = std::max(thr, std::max(tail_l, tail_s));
+    if (ranked) ranked->emplace_back(cost, i);
     if (cost < best) { best = cost; best_i = i; pl->thr = thr; pl->tail_s = tail_s; pl->thr_full = thr_full; }
   }
+  if (force >= 0 && force < menu_size() && menu_entry(force).lane == 0) best_i = force;
   pl->cost = best;
   // test hooks: force a menu entry / team size (used by the parity tests to cover every
   // compiled configuration; never needed for correctness)
@@ -420,8 +432,14 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   int64_t n_long_seqs = 0;
   const Split sp = make_split(h, T, &n_long_seqs);
   const int n_long = sp.n_long;
+  // menu entry: forced while tuning, else the measured one for (m, T) if run_batch tuned it
+  int force = h->tune_force;
+  if (force < 0 && h->db == &h->main_db) {
+    const auto it = h->tuned.find({m, T});
+    if (it != h->tuned.end()) force = it->second;
+  }
   Plan pl;
-  int rc = make_plan(h, m, sp, &pl);
+  int rc = make_plan(h, m, sp, &pl, force);
   if (rc) return rc;
   // Long pairs: T-mode (strips along the database sequence) when the query is short enough
   // that team mode would have few query strips to spread over warps; team mode otherwise.
@@ -437,7 +455,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
     // the main launch then only sees the short pairs: plan it for them
     Split ss = sp;
     ss.n_long = 0; ss.long_cols = 0; ss.long_max_cols = 0;
-    rc = make_plan(h, m, ss, &pl);
+    rc = make_plan(h, m, ss, &pl, force);
     if (rc) return rc;
   }
   h->last_cfg = pl.cfg;
@@ -759,6 +777,68 @@ int build_db(sw_handle h, DbState& db, const uint8_t* residues, const int64_t* o
   return SW_OK;
 }
 
+// Autotune (run_batch): the planner's time model ranks the compiled configurations, but its
+// error is up to ~10 % in team mode (profiles/r01_menu_c3.txt) and a few % in group mode
+// (profiles/r01_plan_check*.jsonl).  The first batch that searches a (query length, threshold)
+// on the loaded database with >= kTuneMinCells cells therefore times the model's kTuneTop best
+// candidates, one search each (every configuration computes the same exact scores, so the
+// candidates write the real output), and keeps the fastest for later searches.  SW_AUTOTUNE=0
+// disables it (model choice only); the tuned table is cleared by sw_load_db.
+constexpr double kTuneMinCells = 1e10;
+constexpr int kTuneTop = 5;
+
+int autotune(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq, int32_t* d_out, int32_t T,
+             cudaStream_t user) {
+  if (h->db != &h->main_db || getenv("SW_FORCE_MENU")) return SW_OK;
+  if (const char* f = getenv("SW_AUTOTUNE"))
+    if (!strcmp(f, "0")) return SW_OK;
+  bool forked = false;
+  const double residues = std::accumulate(h->db->sorted_len.begin(), h->db->sorted_len.end(), 0.0);
+  for (int k = 0; k < nq; ++k) {
+    const int m = (int)(qoff[k + 1] - qoff[k]);
+    if ((double)m * residues < kTuneMinCells) continue;
+    int32_t Tk = T;
+    if (Tk == SW_AUTO_THRESHOLD) Tk = (int32_t)std::min<int64_t>(choose_threshold(h, m), INT32_MAX);
+    const std::pair<int, int32_t> key{m, Tk};
+    if (h->tuned.count(key)) continue;
+    // the candidates of the launch enqueue_query plans (short pairs only when T-mode takes
+    // the long ones)
+    Split sp = make_split(h, Tk, nullptr);
+    if (sp.n_long > 0 && m < kTmodeMaxQuery) { sp.n_long = 0; sp.long_cols = 0; sp.long_max_cols = 0; }
+    if (sp.n_long == 0 && sp.n_short == 0) { h->tuned[key] = -1; continue; }
+    std::vector<std::pair<double, int>> ranked;
+    Plan pl;
+    int rc = make_plan(h, m, sp, &pl, -1, &ranked);
+    if (rc) return rc;
+    std::sort(ranked.begin(), ranked.end());
+    if (ranked.size() > (size_t)kTuneTop) ranked.resize(kTuneTop);
+    if (!forked) {   // the queries were uploaded on the caller's stream
+      SW_CUDA(h, cudaEventRecord(h->fork, user));
+      SW_CUDA(h, cudaStreamWaitEvent(h->slots[0].stream, h->fork, 0));
+      forked = true;
+    }
+    float best_ms = 1e30f;
+    int best_i = -1;
+    for (const auto& c : ranked) {
+      h->tune_force = c.second;
+      cudaEvent_t* ev = h->ev.data() + 3 * k;
+      rc = enqueue_query(h, h->slots[0], d_queries + qoff[k], m, d_out + (int64_t)k * h->db->n_seqs, Tk,
+                         h->h_ovf + k, ev);
+      h->tune_force = -1;
+      if (rc) return rc;
+      SW_CUDA(h, cudaEventSynchronize(ev[1]));
+      float ms = 0.f;
+      SW_CUDA(h, cudaEventElapsedTime(&ms, ev[0], ev[1]));
+      if (getenv("SW_DEBUG_PLAN")) fprintf(stderr, "tune m=%d T=%d menu=%d %.3f ms\n", m, (int)Tk, c.second, ms);
+      if (ms < best_ms) { best_ms = ms; best_i = c.second; }
+    }
+    h->tuned[key] = best_i;
+  }
+  if (forked) SW_CUDA(h, cudaStreamSynchronize(h->slots[0].stream));
+  h->stat_long = h->stat_short = h->stat_launches = 0;
+  return SW_OK;
+}
+
 int run_batch(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq, int32_t* d_out, int32_t T,
               cudaStream_t user) {
   h->stat_long = h->stat_short = h->stat_launches = 0;
@@ -784,6 +864,8 @@ int run_batch(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq
     SW_CUDA(h, cudaEventCreate(&e));
     h->ev.push_back(e);
   }
+  rc = autotune(h, d_queries, qoff, nq, d_out, T, user);
+  if (rc) return rc;
   const int ns = std::min(nq, max_streams);
   SW_CUDA(h, cudaEventRecord(h->fork, user));
   for (int k = 0; k < ns; ++k) SW_CUDA(h, cudaStreamWaitEvent(h->slots[k].stream, h->fork, 0));
@@ -876,6 +958,7 @@ int sw_load_db(sw_handle h, const uint8_t* residues, int64_t total_residues, con
   if (rc) return rc;
   h->db = &h->main_db;
   h->main_db.release();
+  h->tuned.clear();
   return build_db(h, h->main_db, residues, offsets, num_seqs, nullptr);
 }
 

@@ -267,7 +267,7 @@ __device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&t)[R], co
 // letters of column j + 1, for the profile of u).  rb_in[-1] must be a neutral entry (0, 0)
 // (the row buffers carry one leading slot, zero-initialised and only ever rewritten with the
 // neutral fill values).  Returns max(best, this lane's H maxima) (packed per Lane).
-template <class L, int GC, int R, bool TEAM>
+template <class L, int GC, int R, bool TEAM, int PUB = 16>
 __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t* prow, int ls, int hi_off,
                                              const uint16_t* __restrict__ cols, int ncols,
                                              int half, int steps, int P, int passes_total,
@@ -357,12 +357,15 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
     if (store_out) rb_out[max(col, -1)] = make_uint2(y_hr, y_f);
     ++col;
   };
-  // team mode: publish this strip's progress when a group crossed a multiple of 16 columns or
-  // reached the last one (release: the row-buffer stores are visible first)
+  // team mode: publish this strip's progress when a group crossed a multiple of PUB columns (16
+  // in team mode, 4 = every group in T-mode) or reached the last one (release: the row-buffer
+  // stores are visible first).  Measured: every group is +5 % on C3 with query 144 in T-mode
+  // (short strips of the query: the next warp's wait is a larger share) but -15 % in team mode
+  // with query 5478 (profiles/r01_pub_granularity.txt).
   auto publish = [&]() {
     if (TEAM && store_out) {
       const int done = col;   // the last lane's columns < col are stored
-      if (done > 0 && ((done & 15) < 4 || done > rlast))
+      if (done > 0 && (PUB == 4 || (done & 15) < 4 || done > rlast))
         st_release_smem(prog_out, pass_tag(P, min(done, rlast + 1)));
     }
   };
@@ -814,7 +817,7 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const ChainConst& 
       }
       __syncwarp();
       const int si = (P + W) % (W + 1), so = P % (W + 1);
-      b = run_pass<L, 32, C, true>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps, P, S,
+      b = run_pass<L, 32, C, true, 4>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps, P, S,
                                        rb + (int64_t)si * p.rb_cols + 1, rb + (int64_t)so * p.rb_cols + 1, prog + si,
                                        prog + so, b);
     }
