@@ -103,6 +103,7 @@ class ClockSampler:
 
 # ------------------------------------------------------------------------------- workload
 DB_DESC = {"C1": "Swiss-Prot-shaped synthetic DB (parity-small)", "C2": "Swiss-Prot-shaped synthetic DB",
+           "C5": "TrEMBL-scale synthetic DB (50M seqs, mean 320), the GPUs' shards of C5_SHARDS",
            "C4": "Swiss-Prot-shaped synthetic DB", "C3": "long-sequence synthetic DB (all > 3072 residues)"}
 
 
@@ -120,6 +121,17 @@ def make_workload(name: str, rank: int, world: int):
         qs = [gen.make_query(L) for L in gen.C2_QUERY_LENGTHS]
         lens = gen.long_lengths(4096 * world, seed=3)
         seed, mat, T = 3, "BLOSUM62", 3072
+    elif name == "C5":
+        # TrEMBL-scale (50M sequences, ~16G residues, BLOSUM45, the 20 benchmark queries): the
+        # GPUs of this run search shards 0..N-1 of the database cut into C5_SHARDS round-robin
+        # shards (8 = the 8-GPU box; default 64 so one GPU's line takes seconds, not minutes)
+        qs = [gen.make_query(L) for L in gen.BENCH_QUERY_LENGTHS]
+        full = gen.sp_lengths(50_000_000, seed=5, mu=5.4270)
+        n_sh = max(world, int(os.environ.get("C5_SHARDS", "64")))
+        order = np.argsort(-full, kind="stable")
+        view = np.sort(np.concatenate([order[r::n_sh] for r in range(world)]))
+        lens = full[view]
+        seed, mat, T = 5, "BLOSUM45", 3072
     else:
         raise SystemExit(f"unknown config {name}")
     sel = gen.shard_indices(lens, rank, world)
@@ -395,7 +407,8 @@ def bench_ours(args, rank, world, local_rank):
                    "l2": (f"inputs larger than L2 (device DB ~{2 * db.total_residues / 1e6:.0f} MB > 126 MB)"
                           if 2 * db.total_residues > 126e6 else
                           f"device DB ~{2 * db.total_residues / 1e6:.0f} MB fits in L2 (small config)"),
-                   "parallelism": f"db-shard x{world}"},
+                   "parallelism": f"db-shard x{world}",
+                   **({"c5_shards": max(world, int(os.environ.get("C5_SHARDS", "64")))} if args.config == "C5" else {})},
         "clocks": clk,
         "e2e": {"value": round(e2e_gcups, 2), "unit": "GCUPS", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "api": "sw_search_batch (blocking, host buffers; DB resident as in PAPER.md L32)"},

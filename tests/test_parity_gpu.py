@@ -316,3 +316,21 @@ def test_auto_threshold_parity(cfg):
         T = sw.last_threshold()
     _assert_equal(out, ref, db, f"auto T={T}")
     assert T >= 0
+
+
+# ------------------------------------------------------------------ C5 recipe (TrEMBL-scale config)
+def test_c5_slice_blosum45_parity():
+    """A 1/20000 round-robin slice of C5 (50M sequences, mean length 320, BLOSUM45 10/2, the
+    benchmark query lengths): full parity against the oracle for three of the 20 queries."""
+    full = gen.sp_lengths(50_000_000, seed=5, mu=5.4270)
+    order = np.argsort(-full, kind="stable")
+    view = np.sort(order[::20000])
+    lens = full[view]
+    qs = [gen.make_query(L) for L in gen.BENCH_QUERY_LENGTHS]
+    db = gen.build_database(lens, 5, qs)
+    assert db.num_seqs == 2500 and lens.max() == full.max()
+    for m in (144, 1000, 5478):
+        q = gen.make_query(m)
+        ref = _oracle(q, BLOSUM45, 10, 2, db)
+        out, _ = _gpu(q, BLOSUM45, 10, 2, db, 3072)
+        _assert_equal(out, ref, db, f"C5 slice m={m}")

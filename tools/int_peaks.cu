@@ -112,7 +112,10 @@ __device__ __forceinline__ uint32_t prmt_imm(uint32_t a, uint32_t b) {
 }
 constexpr int CM_R = 32;
 constexpr int CM_COLS = 256;
-template <int R, int NT>
+// SH = 1: the engine's step boundary as well (lane chain: (H, F + rho) and the residue pair
+// arrive by __shfl_up_sync, lane 0 takes them from the stream, the profile address depends
+// on the shuffled residues)
+template <int R, int NT, int SH = 0>
 __global__ void __launch_bounds__(NT) k_cellmix(uint32_t* out, uint32_t seed, Rec* rec) {
   uint32_t t[R], e[R];
   const uint32_t nsig = 0xFFFEFFFEu, nrho = 0xFFF6FFF6u, prho = 0x000A000Au;
@@ -129,8 +132,15 @@ __global__ void __launch_bounds__(NT) k_cellmix(uint32_t* out, uint32_t seed, Re
   const int lane = threadIdx.x & 31;
   long long t0 = clock64();
   unsigned long long g0 = gtimer();
+  uint32_t y_res = 0;
   for (int col = 0; col < ITERS / 4; ++col) {
-    const uint32_t res = sres[col & (CM_COLS - 1)];
+    uint32_t res = sres[col & (CM_COLS - 1)];
+    if constexpr (SH) {
+      uint32_t x_hr = __shfl_up_sync(0xffffffffu, hup0, 1), x_f = __shfl_up_sync(0xffffffffu, fs0, 1);
+      uint32_t x_res = __shfl_up_sync(0xffffffffu, y_res, 1);
+      if (lane == 0) { x_hr = 0u; x_f = 0u; x_res = res; }
+      hup0 = x_hr; fs0 = x_f; y_res = x_res; res = x_res;
+    }
     const uint4* plo = reinterpret_cast<const uint4*>(sprof + ((res & 15) * R * 32)) + lane;
     const uint4* phi = reinterpret_cast<const uint4*>(sprof + ((res >> 4) * R * 32)) + lane;
     uint32_t wlo[R / 4], whi[R / 4];
@@ -257,6 +267,8 @@ int main() {
   // the same mix at 3 warps per scheduler (the engine's 384-thread configurations), R = 32 / 48
   run("cellmix_cells_R32_384", k_cellmix<32, 384>, (ITERS / 4) * 32 * 2.0, 384, d_out, d_rec, false);
   run("cellmix_cells_R48_384", k_cellmix<48, 384>, (ITERS / 4) * 48 * 2.0, 384, d_out, d_rec, false);
+  run("cellmix_shfl_R48_384", k_cellmix<48, 384, 1>, (ITERS / 4) * 48 * 2.0, 384, d_out, d_rec, false);
+  run("cellmix_shfl_R32_512", k_cellmix<32, 512, 1>, (ITERS / 4) * 32 * 2.0, 512, d_out, d_rec, false);
   g_rate = mix_rate;
   printf(", \"cells_per_clk_per_gpu\": %.2f, \"sm_mhz_during\": %.0f, \"what\": \"rates = warp-instructions (cellmix: "
          "warp-cells) per SM clock over the per-SM window in which the blocks ran; cells_per_clk_per_gpu = 32 lanes x "
