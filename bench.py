@@ -365,7 +365,7 @@ def bench_ours(args, rank, world, local_rank):
     achieved = cells_local / (kern_ms / 1e3) / 1e9 if kern_ms > 0 else None
     roof = {"bound": "alu", "unit": "GCUPS", "achieved": round(achieved, 2) if achieved else None,
             "peak": None, "frac": None, "traffic": None,
-            "kernel": "k_search (fused inter/intra-task); cells of the 5 launches of one step / their summed "
+            "kernel": f"k_search (fused inter/intra-task); cells of the {nq} launches of one step / their summed "
                       "CUDA-event durations, launches serialised on one stream"}
     if peaks and achieved:
         f_mhz = clk.get("sm_mhz") or peaks.get("sm_mhz_during") or 1965.0

@@ -1,19 +1,30 @@
 """Run tools/int_peaks (GPU) and write MEASURED_INT_PEAKS.json: the measured unit rates, the
 measured cell-mix rate and the derived ALU-pipe bound of the engine's cell update.
-usage (under gpurun): python tools/update_int_peaks.py"""
+usage (under gpurun): python tools/update_int_peaks.py [int_peaks_output.json]"""
 import json
 import os
 import subprocess
+import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 EXE = os.path.join(ROOT, "tools", "int_peaks")
 SRC = EXE + ".cu"
 
-if not os.path.exists(EXE) or os.path.getmtime(EXE) < os.path.getmtime(SRC):
-    subprocess.run(["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-o", EXE, SRC], check=True)
-d = json.loads(subprocess.run([EXE], check=True, capture_output=True, text=True).stdout)
-mix = d.pop("cells_per_clk_per_gpu")
+if len(sys.argv) > 1:          # a saved int_peaks run
+    d = json.load(open(sys.argv[1]))
+else:
+    if not os.path.exists(EXE) or os.path.getmtime(EXE) < os.path.getmtime(SRC):
+        subprocess.run(["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-o", EXE, SRC], check=True)
+    d = json.loads(subprocess.run([EXE], check=True, capture_output=True, text=True).stdout)
+d.pop("cells_per_clk_per_gpu", None)
+# the measured mix: the fastest cell-mix variant (512 or 384 threads, with or without the lane
+# chain's shuffle step boundary), in cells per clock per GPU = warp-cells/clk/SM x 32 x SMs
+mixes = {k: v["warp_instr_per_clk_per_sm"] * 32 * d["sms"] for k, v in d.items()
+         if isinstance(v, dict) and k.startswith("cellmix")}
+best_mix = max(mixes, key=mixes.get)
+mix = round(mixes[best_mix], 2)
 d["measured_mix_cells_per_clk_per_gpu"] = mix
+d["measured_mix_variant"] = best_mix
 alu = 2.0        # warp-instructions / clk / SM on the ALU pipe (4 SMSPs x 16 lanes / 32)
 ops = 4.5        # ALU-pipe instructions per cell pair of sw_engine.cuh cell_rows
 d["derived"] = {
