@@ -116,6 +116,7 @@ struct sw_handle_s {
   // autotune; -1 = keep the model's choice); cleared by sw_load_db
   std::map<std::pair<int, int32_t>, int> tuned;
   int tune_force = -1;            // menu entry forced while tuning / from the tuned table
+  std::vector<uint32_t> qmask;    // letters present in each query of the current batch
   // scratch
   std::vector<QuerySlot> slots;
   int32_t* d_scores_tmp = nullptr;
@@ -425,7 +426,7 @@ int64_t choose_threshold(sw_handle h, int m) {
 }
 
 // Enqueue one query (device query pointer) on slot s; scores to d_out (device, caller order).
-int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t* d_out, int32_t T,
+int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t qmask, int32_t* d_out, int32_t T,
                   int32_t* h_ovf, cudaEvent_t* ev) {
   if (T == SW_AUTO_THRESHOLD) T = (int32_t)std::min<int64_t>(choose_threshold(h, m), INT32_MAX);
   h->last_threshold = T;
@@ -491,8 +492,12 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
   if (rc) return rc;
 
   const int qcols = (int)round_up(m, 8);
-  const int wp_bytes = (int)round_up((int64_t)(h->A + 1) * 32, 128);
-  const int per_warp = 2 * (h->A + 1) * 32 * kTmodeC;
+  // T-mode strip tables hold one row per letter PRESENT in the query plus the pad row (the
+  // query stream carries compact letter indices): 21 rows for a 20-letter query instead of 25,
+  // so more warps fit in shared memory
+  const int a_used = __builtin_popcount(qmask);
+  const int wp_bytes = (int)round_up((int64_t)(a_used + 1) * 32, 128);
+  const int per_warp = 2 * (a_used + 1) * 32 * kTmodeC;
   int t_warps = std::min(kTmodeThreads / 32, (kMaxProfileSmem - wp_bytes) / per_warp);
   if (t_warps < 1) use_t = false;
   int t_grid = 0;
@@ -556,7 +561,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
     // T-mode runs on the slot's second stream, concurrently with the group launch: its CTAs
     // take every SM first (launched first), and as they run out of long pairs the group
     // launch's CTAs take their SMs, so the longest long pair overlaps the short-pair work.
-    SW_CUDA(h, launch_qpair(s.d_qpair, d_q, m, qcols + kPadCols, h->A, st));
+    SW_CUDA(h, launch_qpair(s.d_qpair, d_q, m, qcols + kPadCols, qmask, st));
     SW_CUDA(h, cudaEventRecord(s.fork, st));
     SW_CUDA(h, cudaStreamWaitEvent(s.aux, s.fork, 0));
     TParams t{};
@@ -566,6 +571,8 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
     t.sigma = h->sigma;
     t.max_w = h->max_w;
     t.pad_letter = h->A;
+    t.qmask = qmask;
+    t.A_used = a_used;
     t.qpair = s.d_qpair;
     t.qcols = qcols;
     t.cols = h->db->d_cols;
@@ -599,7 +606,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, int32_t*
       double best_est = 1e300;
       int bestW = 1, best_big = 1 << 30;
       // (single-warp teams measured slower than the model says: not considered)
-      for (int W = std::min(2, t_warps); W <= t_warps; W *= 2) {
+      for (int W = std::min(2, t_warps); W <= t_warps; ++W) {
         if (t_warps % W) continue;
         for (int phase1 = 0; phase1 < 2; ++phase1) {
           if (phase1 && W == t_warps) continue;
@@ -822,7 +829,7 @@ int autotune(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq,
     for (const auto& c : ranked) {
       h->tune_force = c.second;
       cudaEvent_t* ev = h->ev.data() + 3 * k;
-      rc = enqueue_query(h, h->slots[0], d_queries + qoff[k], m, d_out + (int64_t)k * h->db->n_seqs, Tk,
+      rc = enqueue_query(h, h->slots[0], d_queries + qoff[k], m, h->qmask[k], d_out + (int64_t)k * h->db->n_seqs, Tk,
                          h->h_ovf + k, ev);
       h->tune_force = -1;
       if (rc) return rc;
@@ -839,8 +846,8 @@ int autotune(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq,
   return SW_OK;
 }
 
-int run_batch(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq, int32_t* d_out, int32_t T,
-              cudaStream_t user) {
+int run_batch(sw_handle h, const uint8_t* h_queries, const uint8_t* d_queries, const int64_t* qoff, int nq,
+              int32_t* d_out, int32_t T, cudaStream_t user) {
   h->stat_long = h->stat_short = h->stat_launches = 0;
   h->stat_recomputed = -1;
   h->stat_nq = nq;
@@ -864,6 +871,10 @@ int run_batch(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq
     SW_CUDA(h, cudaEventCreate(&e));
     h->ev.push_back(e);
   }
+  // letters present in each query (T-mode builds its strip tables for these only)
+  h->qmask.assign(nq, 0u);
+  for (int k = 0; k < nq; ++k)
+    for (int64_t i = qoff[k]; i < qoff[k + 1]; ++i) h->qmask[k] |= 1u << h_queries[i];
   rc = autotune(h, d_queries, qoff, nq, d_out, T, user);
   if (rc) return rc;
   const int ns = std::min(nq, max_streams);
@@ -871,7 +882,8 @@ int run_batch(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq
   for (int k = 0; k < ns; ++k) SW_CUDA(h, cudaStreamWaitEvent(h->slots[k].stream, h->fork, 0));
   for (int k = 0; k < nq; ++k) {
     QuerySlot& s = h->slots[k % ns];
-    rc = enqueue_query(h, s, d_queries + qoff[k], (int)(qoff[k + 1] - qoff[k]), d_out + (int64_t)k * h->db->n_seqs, T,
+    rc = enqueue_query(h, s, d_queries + qoff[k], (int)(qoff[k + 1] - qoff[k]), h->qmask[k],
+                       d_out + (int64_t)k * h->db->n_seqs, T,
                        h->h_ovf + k, h->ev.data() + 3 * k);
     if (rc) return rc;
   }
@@ -1075,7 +1087,7 @@ int sw_search_stream(sw_handle h, const uint8_t* queries, const int64_t* q_offse
     h->db = &ss.db;
     h->h_ovf = ss.h_ovf;
     h->h_ovf_cap = ss.ovf_cap;
-    rc = run_batch(h, h->d_batch_q, qo.data(), nq, ss.d_sc, length_threshold, st);
+    rc = run_batch(h, queries, h->d_batch_q, qo.data(), nq, ss.d_sc, length_threshold, st);
     h->db = &h->main_db;
     if (rc) break;
     stat_long += h->stat_long; stat_short += h->stat_short; stat_launches += h->stat_launches;
@@ -1120,7 +1132,7 @@ int sw_search_batch_async(sw_handle h, const uint8_t* queries, const int64_t* q_
   if (rc) return rc;
   h->batch_q_cap = (int64_t)cap;
   if (tot > 0) SW_CUDA(h, cudaMemcpyAsync(h->d_batch_q, queries, (size_t)tot, cudaMemcpyHostToDevice, st));
-  return run_batch(h, h->d_batch_q, q_offsets, num_queries, d_scores_out, length_threshold, st);
+  return run_batch(h, queries, h->d_batch_q, q_offsets, num_queries, d_scores_out, length_threshold, st);
 }
 
 int sw_search_async(sw_handle h, int32_t* d_scores_out, int32_t length_threshold, void* cuda_stream) {

@@ -767,7 +767,8 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const ChainConst& 
   constexpr int CB = chunk_bytes<C>();
   constexpr int LS = 32 * C;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int A1 = p.A + 1;
+  const int A1 = p.A_used + 1;                 // compact query letters + the pad row
+  const uint32_t db_pad = (uint32_t)p.pad_letter * 0x101u;
   const int qsteps = (p.qcols + 32 + 3) & ~3;
   int pending = first_item;
   for (;;) {
@@ -796,7 +797,7 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const ChainConst& 
 #pragma unroll
       for (int r = 0; r < C; ++r) {
         const int pos = P * LS + lane * C + r;
-        dp[r] = pos < ncols ? (uint32_t)cp[pos] : c.padpair;
+        dp[r] = pos < ncols ? (uint32_t)cp[pos] : db_pad;
       }
       for (int a = 0; a < A1; ++a) {
         const int8_t* wrow = wp + a * 32;
@@ -848,15 +849,17 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   __shared__ uint32_t sred[kWarps];
   __shared__ int32_t sitem[kWarps];
   __shared__ int32_t sparked;
-  const int A1 = p.A + 1;
+  // rows = the query's letters in compact order (row k = the k-th set bit of qmask) + the pad
+  // row; columns = database letters (the database pad letter A maps to the pad value)
+  const int A1 = p.A_used + 1;
   const int table_bytes = 2 * A1 * LS;        // lo + hi tables of one warp
-  int8_t* wp = reinterpret_cast<int8_t*>(smem);  // (A+1) x 32: w + rho, pad -> -128
+  int8_t* wp = reinterpret_cast<int8_t*>(smem);  // (A_used+1) x 32: w + rho, pad -> -128
   uint8_t* tables = smem + ((A1 * 32 + 127) & ~127);
   const int warp = threadIdx.x >> 5;
   for (int t = threadIdx.x; t < A1 * 32; t += blockDim.x) {
     const int a = t >> 5, d = t & 31;
     int v = kPadValue;
-    if (a < p.A && d < p.A) v = (int)p.matrix[a * p.A + d] + p.rho;
+    if (a < p.A_used && d < p.A) v = (int)p.matrix[(int)__fns(p.qmask, 0, a + 1) * p.A + d] + p.rho;
     wp[t] = (int8_t)v;
   }
   if (threadIdx.x == 0) sparked = -1;
@@ -865,7 +868,7 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   ChainConst c;
   c.rho = p.rho;
   c.sigma = p.sigma;
-  c.padpair = (uint32_t)p.pad_letter | ((uint32_t)p.pad_letter << 8);
+  c.padpair = (uint32_t)p.A_used * 0x101u;     // the query stream's (compact) pad letter
   c.hi_mul = p.hi_mul;
   uint8_t* tab = tables + warp * table_bytes;
   uint2* rb_cta = p.rb + (int64_t)blockIdx.x * (2 * p.warps) * p.rb_cols;

@@ -124,11 +124,13 @@ struct TParams {
   int big_strips;            // phase 1 (one team of all warps) keeps pairs with >= big_strips strips
   uint2* rb; int64_t rb_cols;   // per CTA: 2 * warps slots (teams x (team_warps + 1) <= 2 * warps)
   uint32_t hi_mul;           // 1 << 24 (see SearchParams::hi_mul)
+  uint32_t qmask;            // letters present in the query (bit a = letter code a)
+  int A_used;                // popcount(qmask): compact letter k = the k-th set bit; pad = A_used
 };
 
 cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st);
 cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm);
-cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, int pad, cudaStream_t st);
+cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, uint32_t qmask, cudaStream_t st);
 
 // Traceback of one pair (sw_traceback.cu): dir = m*n bytes, scratch = 7*m ints, result = 6 ints.
 cudaError_t launch_traceback(const uint8_t* q, int m, const uint16_t* dcols, int half, int n, const int8_t* W, int A,

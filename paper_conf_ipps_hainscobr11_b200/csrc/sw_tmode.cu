@@ -5,16 +5,19 @@
 
 namespace swb {
 
-// qpair[i] = q_i | q_i << 8 for i < m, the pad letter pair beyond (qcols + kPadCols entries)
-__global__ void k_qpair(uint16_t* __restrict__ out, const uint8_t* __restrict__ q, int m, int n, int pad) {
+// qpair[i] = c_i | c_i << 8 for i < m, with c_i the compact index of q_i among the letters
+// present in the query (qmask), and the compact pad (popcount(qmask)) beyond (qcols + kPadCols
+// entries)
+__global__ void k_qpair(uint16_t* __restrict__ out, const uint8_t* __restrict__ q, int m, int n, uint32_t qmask) {
+  const int pad = __popc(qmask);
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
-    const int a = i < m ? (int)q[i] : pad;
+    const int a = i < m ? __popc(qmask & ((1u << q[i]) - 1u)) : pad;
     out[i] = (uint16_t)(a | (a << 8));
   }
 }
 
-cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, int pad, cudaStream_t st) {
-  k_qpair<<<(n + 255) / 256, 256, 0, st>>>(out, q, m, n, pad);
+cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, uint32_t qmask, cudaStream_t st) {
+  k_qpair<<<(n + 255) / 256, 256, 0, st>>>(out, q, m, n, qmask);
   return cudaGetLastError();
 }
 
