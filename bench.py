@@ -317,13 +317,15 @@ def bench_ours(args, rank, world, local_rank):
         ms = float(t.item())
 
     # end-to-end through the blocking host API (queries H2D, scores D2H), rank-local + max
-    e2e_steps = max(1, min(args.steps, 3))
-    t0 = time.perf_counter()
-    for _ in range(e2e_steps):
+    # (per-step host wall times, median: one step's time is not skewed by unrelated host load)
+    e2e_times = []
+    for _ in range(max(1, args.steps)):
+        t0 = time.perf_counter()
         host = sw.search_batch(qs, T)
         if dist_on:
             dist.barrier()
-    e2e_s = (time.perf_counter() - t0) / e2e_steps
+        e2e_times.append(time.perf_counter() - t0)
+    e2e_s = float(np.median(e2e_times))
     if dist_on:
         t = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
