@@ -37,6 +37,10 @@ struct QuerySlot {
   size_t rb_t_cap = 0;
   uint16_t* d_qpair = nullptr;    // T-mode query stream
   size_t qpair_cap = 0;
+  int32_t* d_gang = nullptr;      // T-mode gangs: counter, maxima, done counts, progress flags
+  size_t gang_cap = 0;
+  uint2* d_grb = nullptr;         // T-mode gangs: row buffers
+  size_t grb_cap = 0;
   cudaStream_t stream = nullptr;
   cudaStream_t aux = nullptr;      // T-mode launch, concurrent with the group launch
   cudaEvent_t done = nullptr;
@@ -627,6 +631,65 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
       t.team_warps = W;
       t.big_strips = best_big;
       if (const char* f = getenv("SW_T_BIG")) t.big_strips = std::max(1, atoi(f));
+      // Gangs (k_search_t phase 0): when the long pairs are not
+      // hidden under a larger short-pair launch, a pair whose time alone exceeds the launch's
+      // throughput estimate is spread over K CTAs x W warps (one warp per scheduler, the
+      // CTA's other warps wait) until it reaches its wavefront bound ((S - 1) lag + qsteps).
+      const int WG = std::min(4, t_warps);   // gang warps per CTA: one per scheduler
+      t.gang_items = 0; t.gang_ctas = 1; t.gang_warps = WG;
+      {
+        constexpr int kMaxGangItems = 64, kMaxGangCtas = 8;
+        double t_thr = 0.0;
+        for (int pp = 0; pp < n_long; ++pp) {
+          const double S = std::ceil((double)h->db->h_pair_ncols[pp] / spos);
+          t_thr += S * qsteps / util(W, S);
+        }
+        t_thr /= nw;
+        const bool hidden = (double)sp.short_cols > 0.5 * (double)sp.long_cols;
+        int K = 0, items = 0;
+        if (!hidden) {
+          for (int pp = 0; pp < n_long && pp < kMaxGangItems; ++pp) {
+            const double S = std::ceil((double)h->db->h_pair_ncols[pp] / spos);
+            const double alone = item_time(S >= t.big_strips ? t_warps : W, S);
+            if (alone <= 1.15 * t_thr || S < 2.0 * W) break;
+            const double goal = std::max(1.15 * t_thr, 1.05 * ((S - 1.0) * lag + qsteps));
+            int k = 2;
+            while (k < kMaxGangCtas && item_time(k * WG, S) > goal) ++k;
+            K = std::max(K, k);
+            ++items;
+          }
+          while (items > 0 && items * K > t_grid / 2) --items;
+        }
+        if (const char* f = getenv("SW_T_GANG")) {   // tests: "K" or "K:items"
+          K = atoi(f);
+          const char* comma = strchr(f, ':');
+          items = comma ? atoi(comma + 1) : n_long;
+          items = std::min(items, std::min(n_long, t_grid / std::max(1, K)));
+        }
+        if (getenv("SW_DEBUG_PLAN"))
+          fprintf(stderr, "tmode m=%d long_pairs=%d W=%d t_warps=%d big=%d thr=%.0f steps gangs=%d x %d CTAs\n", m,
+                  n_long, W, t_warps, t.big_strips, t_thr, items, K);
+        if (items > 0 && K >= 2) {
+          t.gang_items = items;
+          t.gang_ctas = K;
+          t.big_strips = 1 << 30;
+        }
+      }
+    }
+    if (t.gang_items > 0) {
+      const int GW = t.gang_ctas * t.gang_warps;
+      const size_t ints = 1 + 3 * (size_t)t.gang_items + (size_t)t.gang_items * (GW + 1);
+      rc = grow(h, &s.d_gang, &s.gang_cap, ints * sizeof(int32_t), "alloc gang scratch", s.aux);
+      if (rc) return rc;
+      rc = grow(h, &s.d_grb, &s.grb_cap, (size_t)t.gang_items * (GW + 1) * (qcols + kPadCols + 1) * sizeof(uint2),
+                "alloc gang row buffers", s.aux, true);
+      if (rc) return rc;
+      SW_CUDA(h, cudaMemsetAsync(s.d_gang, 0, ints * sizeof(int32_t), s.aux));
+      t.gang_ctr = s.d_gang;
+      t.gbest = s.d_gang + 1;
+      t.gdone = s.d_gang + 1 + 2 * t.gang_items;
+      t.gprog = reinterpret_cast<uint32_t*>(s.d_gang + 1 + 3 * t.gang_items);
+      t.grb = s.d_grb;
     }
     t.rb = s.d_rb_t;
     t.rb_cols = qcols + kPadCols + 1;
@@ -1242,6 +1305,7 @@ void sw_destroy(sw_handle h) {
     if (s.stream) cudaStreamSynchronize(s.stream);
     cudaFree(s.d_prof); cudaFree(s.d_work); cudaFree(s.d_ovf_count); cudaFree(s.d_ovf_list);
     cudaFree(s.d_rb_group); cudaFree(s.d_rb_team); cudaFree(s.d_query); cudaFree(s.d_rb_t); cudaFree(s.d_qpair);
+    cudaFree(s.d_gang); cudaFree(s.d_grb);
     if (s.stream) cudaStreamDestroy(s.stream);
     if (s.aux) { cudaStreamSynchronize(s.aux); cudaStreamDestroy(s.aux); }
     if (s.fork) cudaEventDestroy(s.fork);

@@ -141,6 +141,15 @@ __device__ __forceinline__ uint32_t ld_acquire_smem(const uint32_t* p) {
 __device__ __forceinline__ void st_release_smem(uint32_t* p, uint32_t v) {
   asm volatile("st.release.cta.shared::cta.u32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
 }
+// gpu-scope flags in global memory (T-mode gangs: a strip pipeline across CTAs)
+__device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
 __device__ __forceinline__ void team_bar(int team, int W) {
   if (W > 1) {
     asm volatile("bar.sync %0, %1;" ::"r"(team + 1), "r"(W * 32) : "memory");
@@ -267,7 +276,7 @@ __device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&t)[R], co
 // letters of column j + 1, for the profile of u).  rb_in[-1] must be a neutral entry (0, 0)
 // (the row buffers carry one leading slot, zero-initialised and only ever rewritten with the
 // neutral fill values).  Returns max(best, this lane's H maxima) (packed per Lane).
-template <class L, int GC, int R, bool TEAM, int PUB = 16>
+template <class L, int GC, int R, bool TEAM, int PUB = 16, bool GPU_FLAGS = false>
 __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t* prow, int ls, int hi_off,
                                              const uint16_t* __restrict__ cols, int ncols,
                                              int half, int steps, int P, int passes_total,
@@ -318,7 +327,7 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
       if constexpr (TEAM) {
         const uint32_t need = pass_tag(P - 1, min(c0 + 3, rlast) + 1);
         while (known < need) {
-          known = ld_acquire_smem(prog_in);
+          known = GPU_FLAGS ? ld_acquire_gpu(prog_in) : ld_acquire_smem(prog_in);
           if (known < need) __nanosleep(32);
         }
       }
@@ -360,13 +369,16 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
   // team mode: publish this strip's progress when a group crossed a multiple of PUB columns (16
   // in team mode, 4 = every group in T-mode) or reached the last one (release: the row-buffer
   // stores are visible first).  Measured: every group is +5 % on C3 with query 144 in T-mode
-  // (short strips of the query: the next warp's wait is a larger share) but -15 % in team mode
-  // with query 5478 (profiles/r01_pub_granularity.txt).
+  // (short sweeps of the query: the next warp's wait is a larger share of each strip,
+  // profiles/r01_pub_granularity.txt); team mode keeps 16.
   auto publish = [&]() {
     if (TEAM && store_out) {
       const int done = col;   // the last lane's columns < col are stored
       if (done > 0 && (PUB == 4 || (done & 15) < 4 || done > rlast))
-        st_release_smem(prog_out, pass_tag(P, min(done, rlast + 1)));
+      {
+        if constexpr (GPU_FLAGS) st_release_gpu(prog_out, pass_tag(P, min(done, rlast + 1)));
+        else st_release_smem(prog_out, pass_tag(P, min(done, rlast + 1)));
+      }
     }
   };
 
@@ -758,6 +770,60 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
 // an item already taken for this team (or -1).  max_strips: a team of W warps only keeps items
 // with at most this many strips (> max_strips: the item is parked in *parked and the loop
 // returns, so that the CTA can regroup into smaller teams for the remaining, shorter items).
+// Build warp's strip tables for strip P of a long pair: position pos = P*LS + lane*C + r;
+// P_lo[a][pos] = w(a, d_lo[pos]) + rho (a = compact query letter), P_hi likewise, chunk-major
+// and lane-private like the query profile (every lane writes and later reads only its chunks).
+template <int C>
+__device__ __forceinline__ void build_strip_tables(const TParams& p, uint8_t* tab, const int8_t* wp,
+                                                   const uint16_t* cp, int ncols, int P) {
+  constexpr int CB = chunk_bytes<C>();
+  constexpr int LS = 32 * C;
+  const int lane = threadIdx.x & 31;
+  const int A1 = p.A_used + 1;
+  const uint32_t db_pad = (uint32_t)p.pad_letter * 0x101u;
+  __syncwarp();
+  uint32_t dp[C];
+#pragma unroll
+  for (int r = 0; r < C; ++r) {
+    const int pos = P * LS + lane * C + r;
+    dp[r] = pos < ncols ? (uint32_t)cp[pos] : db_pad;
+  }
+  for (int a = 0; a < A1; ++a) {
+    const int8_t* wrow = wp + a * 32;
+#pragma unroll
+    for (int k = 0; k < C / 4; ++k) {
+      uint32_t lo = 0, hi = 0;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint32_t d = dp[4 * k + j];
+        lo |= (uint32_t)(uint8_t)wrow[d & 0xff] << (8 * j);
+        hi |= (uint32_t)(uint8_t)wrow[d >> 8] << (8 * j);
+      }
+      const int r0 = 4 * k;
+      const int off = a * LS + ((r0 / CB) * 32 + lane) * CB + (r0 % CB);
+      *reinterpret_cast<uint32_t*>(tab + off) = lo;
+      *reinterpret_cast<uint32_t*>(tab + A1 * LS + off) = hi;
+    }
+  }
+  __syncwarp();
+}
+
+// scores of long pair `item` from its reduced s16x2 maximum (or its overflow flags)
+__device__ __forceinline__ void emit_t(const TParams& p, uint32_t bb, int item) {
+  const int limit = 32767 - p.max_w;
+  const int s0 = 2 * item, s1 = 2 * item + 1;
+  const int lo = (int)(int16_t)(bb & 0xffffu), hi = (int)(int16_t)(bb >> 16);
+  if (lo >= limit) p.ovf_list[atomicAdd(p.ovf_count, 1)] = s0; else p.scores[p.perm[s0]] = lo;
+  if (s1 < p.n_seqs) {
+    if (hi >= limit) p.ovf_list[atomicAdd(p.ovf_count, 1)] = s1; else p.scores[p.perm[s1]] = hi;
+  }
+}
+
+// One T-mode team (W warps) processing long pairs until the queue is exhausted.  first_item:
+// an item already taken for this team (or -1).  min_strips: a team of W warps only keeps items
+// with at least this many strips (fewer: the item is parked in *parked and the loop returns,
+// so that the CTA can regroup into smaller teams for the remaining, shorter items).  Items
+// [0, gang_items) belong to the gangs (t_gang_item); the queue starts after them.
 template <int C>
 __device__ __forceinline__ void t_team_loop(const TParams& p, const ChainConst& c, uint8_t* tab,
                                             const int8_t* wp, int W, int team, int wt, int first_item,
@@ -768,13 +834,12 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const ChainConst& 
   constexpr int LS = 32 * C;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int A1 = p.A_used + 1;                 // compact query letters + the pad row
-  const uint32_t db_pad = (uint32_t)p.pad_letter * 0x101u;
   const int qsteps = (p.qcols + 32 + 3) & ~3;
   int pending = first_item;
   for (;;) {
     team_bar(team, W);
     if (wt == 0 && lane == 0) {
-      const int it = pending >= 0 ? pending : atomicAdd(p.work, 1);
+      const int it = pending >= 0 ? pending : p.gang_items + atomicAdd(p.work, 1);
       sitem[team] = it;
       for (int i = 0; i <= W; ++i) prog[i] = 0u;
     }
@@ -791,32 +856,7 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const ChainConst& 
     const uint16_t* cp = p.cols + p.pair_off[item];
     uint32_t b = 0;
     for (int P = wt; P < S; P += W) {
-      // build this warp's strip tables: position pos = P*LS + lane*C + r
-      __syncwarp();
-      uint32_t dp[C];
-#pragma unroll
-      for (int r = 0; r < C; ++r) {
-        const int pos = P * LS + lane * C + r;
-        dp[r] = pos < ncols ? (uint32_t)cp[pos] : db_pad;
-      }
-      for (int a = 0; a < A1; ++a) {
-        const int8_t* wrow = wp + a * 32;
-#pragma unroll
-        for (int k = 0; k < C / 4; ++k) {
-          uint32_t lo = 0, hi = 0;
-#pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            const uint32_t d = dp[4 * k + j];
-            lo |= (uint32_t)(uint8_t)wrow[d & 0xff] << (8 * j);
-            hi |= (uint32_t)(uint8_t)wrow[d >> 8] << (8 * j);
-          }
-          const int r0 = 4 * k;
-          const int off = a * LS + ((r0 / CB) * 32 + lane) * CB + (r0 % CB);
-          *reinterpret_cast<uint32_t*>(tab + off) = lo;
-          *reinterpret_cast<uint32_t*>(tab + A1 * LS + off) = hi;
-        }
-      }
-      __syncwarp();
+      build_strip_tables<C>(p, tab, wp, cp, ncols, P);
       const int si = (P + W) % (W + 1), so = P % (W + 1);
       b = run_pass<L, 32, C, true, 4>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps, P, S,
                                        rb + (int64_t)si * p.rb_cols + 1, rb + (int64_t)so * p.rb_cols + 1, prog + si,
@@ -829,13 +869,52 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const ChainConst& 
     if (wt == 0 && lane == 0) {
       uint32_t bb = sred[team * W];
       for (int i = 1; i < W; ++i) bb = L::max2(bb, sred[team * W + i]);
-      const int limit = 32767 - p.max_w;
-      const int s0 = 2 * item, s1 = 2 * item + 1;
-      const int lo = (int)(int16_t)(bb & 0xffffu), hi = (int)(int16_t)(bb >> 16);
-      if (lo >= limit) p.ovf_list[atomicAdd(p.ovf_count, 1)] = s0; else p.scores[p.perm[s0]] = lo;
-      if (s1 < p.n_seqs) {
-        if (hi >= limit) p.ovf_list[atomicAdd(p.ovf_count, 1)] = s1; else p.scores[p.perm[s1]] = hi;
-      }
+      emit_t(p, bb, item);
+    }
+  }
+}
+
+// A GANG: the longest pairs' strips spread over gang_ctas CTAs x gang_warps warps (one warp per
+// scheduler of each SM), so that one 35k-residue sequence is not bound to one SM.  Global warp
+// gw = rank * gang_warps + warp takes strips gw, gw + GW, ...; the strip hand-off is the team
+// pipeline with its row buffers and progress flags in global memory at gpu scope
+// (release / acquire).  The pair's maximum is combined with atomicMax over the GW warps and
+// emitted by the last one.  (Every gang CTA is resident: the T-mode grid is one wave, and a
+// slot's dependencies were taken by CTAs that started earlier.)
+template <int C>
+__device__ __forceinline__ void t_gang_item(const TParams& p, const ChainConst& c, uint8_t* tab, const int8_t* wp,
+                                            int gi, int rank, int warp) {
+  using L = LaneS16x2;
+  constexpr int CB = chunk_bytes<C>();
+  constexpr int LS = 32 * C;
+  const int lane = threadIdx.x & 31;
+  const int A1 = p.A_used + 1;
+  const int qsteps = (p.qcols + 32 + 3) & ~3;
+  const int GW = p.gang_ctas * p.gang_warps;
+  const int gw = rank * p.gang_warps + warp;
+  const int ncols = p.pair_ncols[gi];
+  const int S = (ncols + LS - 1) / LS;
+  const uint16_t* cp = p.cols + p.pair_off[gi];
+  uint2* rb = p.grb + (int64_t)gi * (GW + 1) * p.rb_cols;
+  uint32_t* prog = p.gprog + (int64_t)gi * (GW + 1);
+  uint32_t b = 0;
+  for (int P = gw; P < S; P += GW) {
+    build_strip_tables<C>(p, tab, wp, cp, ncols, P);
+    const int si = (P + GW) % (GW + 1), so = P % (GW + 1);
+    b = run_pass<L, 32, C, true, 16, true>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps, P, S,
+                                          rb + (int64_t)si * p.rb_cols + 1, rb + (int64_t)so * p.rb_cols + 1,
+                                          prog + si, prog + so, b);
+  }
+#pragma unroll
+  for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
+  if (lane == 0) {
+    atomicMax(&p.gbest[2 * gi], (int)(int16_t)(b & 0xffffu));
+    atomicMax(&p.gbest[2 * gi + 1], (int)(int16_t)(b >> 16));
+    __threadfence();
+    if (atomicAdd(&p.gdone[gi], 1) == GW - 1) {   // the last warp of the gang
+      __threadfence();
+      const int lo = atomicAdd(&p.gbest[2 * gi], 0), hi = atomicAdd(&p.gbest[2 * gi + 1], 0);
+      emit_t(p, ((uint32_t)lo & 0xffffu) | ((uint32_t)hi << 16), gi);
     }
   }
 }
@@ -876,7 +955,20 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   // very long ones get the most parallelism; stops at the first pair with few strips.
   // Phase 2: teams of team_warps for the rest — small teams waste less time in the pipeline
   // fill and in the end-of-item barrier (T-mode ncu: 17 % barrier stalls with 8-warp teams).
-  if (p.warps > p.team_warps) {
+  // Phase 0 (gangs): every CTA takes one gang slot; slot s = (pair s / gang_ctas, rank
+  // s % gang_ctas).  The CTA's first gang_warps warps (one per scheduler) work on that pair
+  // while its other warps wait, so that the gang's dependency chain has its schedulers to
+  // itself; then all warps go on to phase 2.
+  if (p.gang_items > 0) {
+    __shared__ int32_t sgslot;
+    if (threadIdx.x == 0) sgslot = atomicAdd(p.gang_ctr, 1);
+    __syncthreads();
+    const int gi = sgslot / p.gang_ctas, rank = sgslot % p.gang_ctas;
+    if (gi < p.gang_items) {
+      if (warp < p.gang_warps) t_gang_item<C>(p, c, tab, wp, gi, rank, warp);
+      __syncthreads();
+    }
+  } else if (p.warps > p.team_warps) {
     t_team_loop<C>(p, c, tab, wp, p.warps, 0, warp, -1, p.big_strips, &sparked, sprog, rb_cta, sitem, sred);
     __syncthreads();
   }

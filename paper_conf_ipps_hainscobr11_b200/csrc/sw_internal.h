@@ -126,6 +126,14 @@ struct TParams {
   uint32_t hi_mul;           // 1 << 24 (see SearchParams::hi_mul)
   uint32_t qmask;            // letters present in the query (bit a = letter code a)
   int A_used;                // popcount(qmask): compact letter k = the k-th set bit; pad = A_used
+  // gangs (k_search_t phase 0): pairs [0, gang_items) are spread over gang_ctas CTAs x
+  // gang_warps warps each; all buffers below are per gang pair and zeroed before the launch
+  int gang_items, gang_ctas, gang_warps;
+  int32_t* gang_ctr;         // slot counter
+  uint32_t* gprog;           // gang_items x (GW + 1) progress flags, GW = gang_ctas * gang_warps
+  uint2* grb;                // gang_items x (GW + 1) x rb_cols row buffers
+  int32_t* gbest;            // gang_items x 2: maxima of the pair's two sequences
+  int32_t* gdone;            // gang_items: warps finished
 };
 
 cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st);

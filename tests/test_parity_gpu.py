@@ -109,6 +109,23 @@ def test_long_sequence_modes(mode, m):
         _assert_equal(out, ref, db, f"mode={mode} m={m} T={T}")
 
 
+@pytest.mark.parametrize("gang", ["2", "3", "8", "2:1", "5:3"])
+@pytest.mark.parametrize("m", [1, 144, 1500])
+def test_tmode_gangs(gang, m):
+    """T-mode gangs: the longest pairs spread over K CTAs (strip pipeline across CTAs through
+    global row buffers and gpu-scope progress flags), SW_T_GANG = "K" (every long pair) or
+    "K:items" (the items longest pairs); the other pairs take the CTA teams."""
+    rng = np.random.default_rng(500 + m)
+    lens = np.concatenate([[35213, 20000, 513, 512, 3073], rng.integers(3000, 15000, size=11),
+                           rng.integers(0, 300, size=9)])
+    db = _db_from_lengths(lens, seed=600 + m, extra=True)
+    q = gen.make_query(m, seed=990 + m)
+    ref = _oracle(q, BLOSUM62, 10, 2, db)
+    for T in (0, 3000):
+        out, _ = _gpu(q, BLOSUM62, 10, 2, db, T, env={"SW_LONG_MODE": "t", "SW_T_GANG": gang})
+        _assert_equal(out, ref, db, f"gang={gang} m={m} T={T}")
+
+
 @pytest.mark.parametrize("team", [1, 2, 3, 5])
 def test_team_mode_multi_warp(team):
     """Intra-task path with several warps chained over strips (progress-flag hand-off)."""
