@@ -102,6 +102,15 @@ int sw_search_batch_async(sw_handle h, const uint8_t* queries, const int64_t* q_
                           int32_t num_queries, int32_t* d_scores_out, int32_t length_threshold,
                           void* cuda_stream);
 
+/* Autotune (all search calls on a database loaded with sw_load_db): the first search of a
+ * (query length, threshold) whose cells (query length x database residues) reach 1e10 times
+ * the planner's 5 best kernel configurations, one search each, on the handle's first internal
+ * stream, and keeps the fastest for later searches of that (query length, threshold).  That
+ * first call therefore synchronises with the device (the async variants block for it) and
+ * costs about five searches; its scores are the exact ones (every configuration computes the
+ * same scores).  The table is cleared by sw_load_db.  Environment SW_AUTOTUNE=0 disables it
+ * (the planner's model choice only). */
+
 /* Host-pointer variant of sw_search_batch_async (blocking; host int32[num_queries*num_seqs]). */
 int sw_search_batch(sw_handle h, const uint8_t* queries, const int64_t* q_offsets,
                     int32_t num_queries, int32_t* scores_out, int32_t length_threshold);
