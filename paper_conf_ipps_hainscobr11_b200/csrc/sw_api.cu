@@ -456,6 +456,8 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     if (!strcmp(f, "team")) use_t = false;
     if (!strcmp(f, "t")) use_t = n_long > 0;
   }
+  // T-mode progress tags hold the query column in 13 bits (sw_engine.cuh t_team_stream)
+  if (round_up(m, 8) + kPadCols + 36 >= 8192) use_t = false;
   if (use_t) {
     // the main launch then only sees the short pairs: plan it for them
     Split ss = sp;

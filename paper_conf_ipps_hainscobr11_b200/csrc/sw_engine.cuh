@@ -214,10 +214,6 @@ __device__ __forceinline__ uint32_t subst_row(const uint32_t (&wlo)[(R + 3) / 4]
   }
 }
 
-__device__ __forceinline__ uint32_t pass_tag(int pass, int cols_done) {
-  return ((uint32_t)pass << 20) | (uint32_t)cols_done;
-}
-
 struct ChainConst {
   int rho, sigma;
   uint32_t padpair;       // residue pair of two pad letters
@@ -276,12 +272,17 @@ __device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&t)[R], co
 // letters of column j + 1, for the profile of u).  rb_in[-1] must be a neutral entry (0, 0)
 // (the row buffers carry one leading slot, zero-initialised and only ever rewritten with the
 // neutral fill values).  Returns max(best, this lane's H maxima) (packed per Lane).
-template <class L, int GC, int R, bool TEAM, int PUB = 16, bool GPU_FLAGS = false>
+template <class L, int GC, int R, bool TEAM, int PUB = 16, bool GPU_FLAGS = false, int TAG_SHIFT = 20>
 __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t* prow, int ls, int hi_off,
                                              const uint16_t* __restrict__ cols, int ncols,
                                              int half, int steps, int P, int passes_total,
                                              const uint2* __restrict__ rb_in, uint2* __restrict__ rb_out,
-                                             const uint32_t* prog_in, uint32_t* prog_out, uint32_t best) {
+                                             const uint32_t* prog_in, uint32_t* prog_out, uint32_t best,
+                                             int tagP = -1) {
+  // progress tags: (strip index << TAG_SHIFT) | columns done, monotonic per flag slot; the
+  // strip index is the pass P, or the team stream's running strip index tagP
+  const uint32_t tag_base = (uint32_t)(tagP >= 0 ? tagP : P) << TAG_SHIFT;
+  const uint32_t tag_prev = tag_base - (1u << TAG_SHIFT);
   static_assert(R % 4 == 0 || R >= 12, "R < 12 must be a multiple of 4");
   const int lane = threadIdx.x & 31;
   const int gl = lane & (GC - 1);
@@ -325,7 +326,7 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
     for (int k = 0; k < 4; ++k) rr[k] = cols[min(c0 + k + 1, cmax)];
     if (from_prev) {
       if constexpr (TEAM) {
-        const uint32_t need = pass_tag(P - 1, min(c0 + 3, rlast) + 1);
+        const uint32_t need = tag_prev | (uint32_t)(min(c0 + 3, rlast) + 1);
         while (known < need) {
           known = GPU_FLAGS ? ld_acquire_gpu(prog_in) : ld_acquire_smem(prog_in);
           if (known < need) __nanosleep(32);
@@ -376,8 +377,8 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
       const int done = col;   // the last lane's columns < col are stored
       if (done > 0 && (PUB == 4 || (done & 15) < 4 || done > rlast))
       {
-        if constexpr (GPU_FLAGS) st_release_gpu(prog_out, pass_tag(P, min(done, rlast + 1)));
-        else st_release_smem(prog_out, pass_tag(P, min(done, rlast + 1)));
+        if constexpr (GPU_FLAGS) st_release_gpu(prog_out, tag_base | (uint32_t)min(done, rlast + 1));
+        else st_release_smem(prog_out, tag_base | (uint32_t)min(done, rlast + 1));
       }
     }
   };
@@ -874,6 +875,104 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const ChainConst& 
   }
 }
 
+// T-mode team STREAM (phase 2): the strips of the pairs a team takes form one running strip
+// sequence g = 0, 1, 2, ... (pair after pair, longest first from the global queue); warp wt of
+// the W-warp team processes g = wt, wt + W, ...  A warp that has finished its strips of one
+// pair goes straight on to the next pair's, so the team's pipeline is filled and drained once
+// per launch instead of once per pair (the per-pair barrier and the (W - 1) x lag fill were
+// ~10-20 % of T-mode time for short queries).  Hand-off and flags are the team pipeline's
+// (slot g mod (W + 1), tag = g): strip g + 1 consumes strip g's bottom row only inside a pair.
+// Each pair's maximum is combined with atomicMax in the team's shared ring of pairs; the
+// warp finishing its last strip emits the scores.
+constexpr int kTQ = 16;      // pairs in a team's ring (a team spans at most ~W + 1 of them)
+struct TStream {
+  int lock, count, next, end;
+  int item[kTQ], base[kTQ], S[kTQ], rem[kTQ], mlo[kTQ], mhi[kTQ];
+};
+
+template <int C>
+__device__ __forceinline__ void t_team_stream(const TParams& p, const ChainConst& c, uint8_t* tab,
+                                              const int8_t* wp, int W, int team, int wt, int first_item,
+                                              uint32_t* prog, uint2* rb, TStream* ts) {
+  using L = LaneS16x2;
+  constexpr int CB = chunk_bytes<C>();
+  constexpr int LS = 32 * C;
+  const int lane = threadIdx.x & 31;
+  const int A1 = p.A_used + 1;
+  const int qsteps = (p.qcols + 32 + 3) & ~3;
+  volatile TStream* vs = ts;
+  // append one pair to the ring (lane 0 of the warp holding the lock); empty pairs score 0
+  auto append = [&](int item) {
+    const int S = (p.pair_ncols[item] + LS - 1) / LS;
+    if (S == 0) { emit_t(p, 0u, item); return; }
+    const int k = vs->count % kTQ;
+    if (vs->count >= kTQ)   // the entry kTQ pairs back must be finished before it is reused
+      while (vs->rem[k] != 0) __nanosleep(64);
+    vs->item[k] = item; vs->base[k] = vs->next; vs->S[k] = S; vs->rem[k] = S; vs->mlo[k] = 0; vs->mhi[k] = 0;
+    __threadfence_block();
+    vs->count = vs->count + 1;
+    vs->next = vs->next + S;
+  };
+  team_bar(team, W);
+  if (wt == 0 && lane == 0) {
+    for (int i = 0; i <= W; ++i) prog[i] = 0u;
+    ts->lock = 0; ts->count = 0; ts->next = 0; ts->end = 0;
+    if (first_item >= 0) append(first_item);
+    __threadfence_block();
+  }
+  team_bar(team, W);
+  for (int g = wt;; g += W) {
+    // the ring entry of strip g (lane 0 decides, the warp follows)
+    int k = -1;
+    if (lane == 0) {
+      for (;;) {
+        const int next = vs->next, count = vs->count;
+        if (g < next) {
+          for (int j = count - 1; j >= 0 && j >= count - kTQ; --j) {
+            const int kk = j % kTQ;
+            if (vs->base[kk] <= g) { k = kk; break; }
+          }
+          break;
+        }
+        if (vs->end) break;
+        if (atomicCAS(&ts->lock, 0, 1) == 0) {
+          while (vs->next <= g && !vs->end) {
+            const int item = p.gang_items + atomicAdd(p.work, 1);
+            if (item >= p.n_items) { vs->end = 1; break; }
+            append(item);
+          }
+          __threadfence_block();
+          atomicExch(&ts->lock, 0);
+        } else {
+          __nanosleep(64);
+        }
+      }
+    }
+    k = __shfl_sync(SWB_FULL, k, 0);
+    if (k < 0) break;
+    const int item = vs->item[k], P = g - vs->base[k], S = vs->S[k];
+    const int ncols = p.pair_ncols[item];
+    const uint16_t* cp = p.cols + p.pair_off[item];
+    build_strip_tables<C>(p, tab, wp, cp, ncols, P);
+    const int si = (g + W) % (W + 1), so = g % (W + 1);
+    uint32_t b = run_pass<L, 32, C, true, 4, false, 13>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps,
+                                                       P, S, rb + (int64_t)si * p.rb_cols + 1,
+                                                       rb + (int64_t)so * p.rb_cols + 1, prog + si, prog + so, 0u, g);
+#pragma unroll
+    for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
+    if (lane == 0) {
+      atomicMax(&ts->mlo[k], (int)(int16_t)(b & 0xffffu));
+      atomicMax(&ts->mhi[k], (int)(int16_t)(b >> 16));
+      __threadfence_block();
+      if (atomicSub(&ts->rem[k], 1) == 1) {   // this pair's last strip
+        const int lo = atomicAdd(&ts->mlo[k], 0), hi = atomicAdd(&ts->mhi[k], 0);
+        emit_t(p, ((uint32_t)lo & 0xffffu) | ((uint32_t)hi << 16), item);
+      }
+    }
+    __syncwarp();
+  }
+}
+
 // A GANG: the longest pairs' strips spread over gang_ctas CTAs x gang_warps warps (one warp per
 // scheduler of each SM), so that one 35k-residue sequence is not bound to one SM.  Global warp
 // gw = rank * gang_warps + warp takes strips gw, gw + GW, ...; the strip hand-off is the team
@@ -977,8 +1076,9 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   const int team = warp / W, wt = warp % W;
   if (team >= nteams) return;
   const int first = (team == 0) ? sparked : -1;
-  t_team_loop<C>(p, c, tab, wp, W, team, wt, first, 0, nullptr, sprog + team * (W + 1),
-                     rb_cta + (int64_t)team * (W + 1) * p.rb_cols, sitem, sred);
+  __shared__ TStream sts[kTmodeThreads / 32];
+  t_team_stream<C>(p, c, tab, wp, W, team, wt, first, sprog + team * (W + 1),
+                   rb_cta + (int64_t)team * (W + 1) * p.rb_cols, &sts[team]);
 }
 
 template <int C, int NT>
