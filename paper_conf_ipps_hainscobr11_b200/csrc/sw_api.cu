@@ -400,9 +400,9 @@ int64_t choose_threshold(sw_handle h, int m) {
     if (!make_plan(h, m, sp, &pl) && sp.short_cols > 0) per_col = pl.thr_full * (2.7 / 2.0) / (double)sp.short_cols;
   }
   // long path cost per column relative to the group path at full occupancy, measured (C3 all
-  // long vs C2 short, profiles/r01_sweep_c3_*.jsonl): 2.4 at m = 144, 1.57 at 567, 1.43 at
-  // 1500, 1.21 at 5478 (linear in between)
-  const double lm[] = {144, 567, 1500, 5478}, lf[] = {2.4, 1.57, 1.43, 1.21};
+  // long vs C2 short-only, profiles/r01_sweep_*.jsonl, with the T-mode team stream): 2.02 at
+  // m = 144, 1.55 at 567, 1.44 at 1500, 1.16 at 5478 (linear in between)
+  const double lm[] = {144, 567, 1500, 5478}, lf[] = {2.02, 1.55, 1.44, 1.16};
   double long_factor = lf[3];
   if (m <= lm[0]) long_factor = lf[0];
   for (int k = 0; k < 3; ++k)
