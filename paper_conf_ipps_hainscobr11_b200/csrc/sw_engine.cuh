@@ -457,12 +457,16 @@ struct GsState {
   uint32_t desc[2];
 };
 
-template <class L, int R>
+// MULTI = false: the query fits one strip (p.short_passes == 1), so there is no strip row
+// buffer: the first lane's top input is the constant boundary (H, F + rho) = (0, 0) and only
+// the residues go through the fetch ring (8 registers and 2 selects per step fewer).
+template <class L, int R, bool MULTI>
 __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainConst& c, const uint8_t* pbase,
                                              uint2* __restrict__ rb, volatile GsState* gs) {
   static_assert(R % 4 == 0 || R >= 12, "R < 12 must be a multiple of 4");
   constexpr int kGap = 4;
   const int lane = threadIdx.x & 31;
+  const uint32_t not0 = lane == 0 ? 0u : 1u;
   const uint32_t nrho = L::splat(-c.rho), prho = L::splat(c.rho);
   const uint32_t nsig = L::splat(-c.sigma);
   constexpr int CB = chunk_bytes<R>();
@@ -547,8 +551,10 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
   uint32_t ring_res[4], ring_h[4], ring_f[4];
   auto fetch = [&](int k) {
     ring_res[k] = g_cols[k];
-    const uint2 v = g_rb[k];
-    ring_h[k] = v.x; ring_f[k] = v.y;
+    if constexpr (MULTI) {
+      const uint2 v = g_rb[k];
+      ring_h[k] = v.x; ring_f[k] = v.y;
+    }
   };
 
   // ---- per-lane state (look-ahead form, cell_rows)
@@ -570,7 +576,12 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
     uint32_t x_hr = __shfl_up_sync(SWB_FULL, y_hr, 1);
     uint32_t x_f = __shfl_up_sync(SWB_FULL, y_f, 1);
     uint32_t x_res = __shfl_up_sync(SWB_FULL, y_res, 1);
-    if (lane == 0) { x_hr = ring_h[K]; x_f = ring_f[K]; x_res = ring_res[K]; }
+    if constexpr (MULTI) {
+      if (lane == 0) { x_hr = ring_h[K]; x_f = ring_f[K]; x_res = ring_res[K]; }
+    } else {
+      x_hr *= not0; x_f *= not0;     // (IMAD: the boundary row is 0 for the first lane)
+      if (lane == 0) x_res = ring_res[K];
+    }
     uint32_t wlo[(R + 3) / 4], whi[(R + 3) / 4];   // profile words of the next position's letters
     {
       // letter offsets with FMA-pipe ops only: a_hi = x >> 8 as IMAD.HI, a_lo = x - 256 a_hi
@@ -602,7 +613,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
       my_pos -= my_len;
       my_len = (int)(d & (uint32_t)kEndLen);
       my_P = (int)(d >> 24) - 1;
-      store_rb = lane == 31 && my_P >= 0 && my_P < passes - 1;
+      store_rb = MULTI && lane == 31 && my_P >= 0 && my_P < passes - 1;
       prow = pbase + max(my_P, 0) * kStripBytes;
 #pragma unroll
       for (int r = 0; r < R; ++r) { e[r] = nrho; t[r] = 0u; }
@@ -720,8 +731,9 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
     if (p.item_list == nullptr && p.group_stream) {
       constexpr int CBs = chunk_bytes<Rs>();
       __shared__ GsState sgs[kWarps];
-      group_stream<L, Rs>(p, c, smem + p.lg.off + lane * CBs,
-                          p.rb_group + (int64_t)(blockIdx.x * kWarps + warp) * p.rb_group_cols + 4, &sgs[warp]);
+      uint2* rbw = p.rb_group + (int64_t)(blockIdx.x * kWarps + warp) * p.rb_group_cols + 4;
+      if (p.short_passes > 1) group_stream<L, Rs, true>(p, c, smem + p.lg.off + lane * CBs, rbw, &sgs[warp]);
+      else group_stream<L, Rs, false>(p, c, smem + p.lg.off + lane * CBs, rbw, &sgs[warp]);
       return;
     }
   }
