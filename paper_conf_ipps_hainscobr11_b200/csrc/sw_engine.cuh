@@ -272,7 +272,10 @@ __device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&t)[R], co
 // letters of column j + 1, for the profile of u).  rb_in[-1] must be a neutral entry (0, 0)
 // (the row buffers carry one leading slot, zero-initialised and only ever rewritten with the
 // neutral fill values).  Returns max(best, this lane's H maxima) (packed per Lane).
-template <class L, int GC, int R, bool TEAM, int PUB = 16, bool GPU_FLAGS = false, int TAG_SHIFT = 20>
+// ONE_PASS: the query is one strip (no row buffer in or out): the first lane's top input is
+// the constant boundary (0, 0), so the boundary rings and their loads disappear (registers).
+template <class L, int GC, int R, bool TEAM, int PUB = 16, bool GPU_FLAGS = false, int TAG_SHIFT = 20,
+          bool ONE_PASS = false>
 __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t* prow, int ls, int hi_off,
                                              const uint16_t* __restrict__ cols, int ncols,
                                              int half, int steps, int P, int passes_total,
@@ -290,8 +293,8 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
   const uint32_t nsig = L::splat(-c.sigma);
   const int hshift = 8 * half;
   constexpr int CB = chunk_bytes<R>();
-  const bool store_out = (gl == GC - 1) && (P < passes_total - 1);
-  const bool from_prev = P > 0;
+  const bool store_out = !ONE_PASS && (gl == GC - 1) && (P < passes_total - 1);
+  const bool from_prev = !ONE_PASS && P > 0;
 
   uint32_t e[R], t[R];
 #pragma unroll
@@ -345,7 +348,13 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
     uint32_t x_hr = __shfl_up_sync(SWB_FULL, y_hr, 1, GC);
     uint32_t x_f = __shfl_up_sync(SWB_FULL, y_f, 1, GC);
     uint32_t x_res = __shfl_up_sync(SWB_FULL, y_res, 1, GC);
-    if (gl == 0) { x_hr = rh[K]; x_f = rf[K]; x_res = rr[K]; }
+    if constexpr (ONE_PASS) {
+      const uint32_t not0 = gl == 0 ? 0u : 1u;
+      x_hr *= not0; x_f *= not0;     // (IMAD: the boundary row is 0 for the first lane)
+      if (gl == 0) x_res = rr[K];
+    } else {
+      if (gl == 0) { x_hr = rh[K]; x_f = rf[K]; x_res = rr[K]; }
+    }
     // query-profile words for the two letters of the NEXT column (look-ahead u)
     uint32_t wlo[(R + 3) / 4], whi[(R + 3) / 4];
     if constexpr (L::kSeqs == 2) {
@@ -753,12 +762,19 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
       const int steps = ((int)__reduce_max_sync(SWB_FULL, (unsigned)ncols) + G + 3) & ~3;
       uint2* rb = p.rb_group + ((int64_t)(blockIdx.x * kWarps + warp) * GPW + gi) * p.rb_group_cols;
       uint32_t b = 0;
-      for (int P = 0; P < p.short_passes; ++P) {
+      if (p.short_passes == 1) {
         constexpr int CBs = chunk_bytes<Rs>();
-        const uint8_t* prow = smem + p.lg.off + gi * p.lg.rs + (P * chunks_per_lane<Rs>() * G + gl) * CBs;
-        b = run_pass<L, G, Rs, false>(c, prow, p.lg.ls, 0, cp, ncols, 0, steps, P, p.short_passes, rb + 1, rb + 1, nullptr,
-                                      nullptr, b);
-        __syncwarp();   // strip P's bottom row (written by lane G-1) is read by lane 0 in strip P+1
+        const uint8_t* prow = smem + p.lg.off + gi * p.lg.rs + gl * CBs;
+        b = run_pass<L, G, Rs, false, 16, false, 20, true>(c, prow, p.lg.ls, 0, cp, ncols, 0, steps, 0, 1, rb + 1,
+                                                            rb + 1, nullptr, nullptr, b);
+      } else {
+        for (int P = 0; P < p.short_passes; ++P) {
+          constexpr int CBs = chunk_bytes<Rs>();
+          const uint8_t* prow = smem + p.lg.off + gi * p.lg.rs + (P * chunks_per_lane<Rs>() * G + gl) * CBs;
+          b = run_pass<L, G, Rs, false>(c, prow, p.lg.ls, 0, cp, ncols, 0, steps, P, p.short_passes, rb + 1, rb + 1,
+                                        nullptr, nullptr, b);
+          __syncwarp();   // strip P's bottom row (written by lane G-1) is read by lane 0 in strip P+1
+        }
       }
 #pragma unroll
       for (int o = G / 2; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
