@@ -49,7 +49,13 @@ enum {
 
 /* Limits (validated; SW_E_INVALID / SW_E_UNSUPPORTED otherwise). */
 #define SW_MAX_ALPHABET 32          /* alphabet_size in [1, 32] */
-#define SW_MAX_QUERY_LEN (1 << 16)  /* 1 <= query_len <= 65536 */
+#define SW_MAX_QUERY_LEN (1 << 16)  /* 1 <= query_len <= 65536 (SW_E_INVALID beyond) */
+/* The int8 query profile (alphabet_size + 1 rows of query_len bytes, padded to the kernel's
+ * strip layout) is staged whole in one CTA's shared memory; a search whose profile exceeds
+ * SW_MAX_PROFILE_BYTES fails with SW_E_UNSUPPORTED (never a CPU fallback).  In practice:
+ * query_len <= 8192 for the 24-letter protein alphabet (the paper's queries reach 5478),
+ * query_len = 65536 for alphabets of up to 2 letters. */
+#define SW_MAX_PROFILE_BYTES (220 * 1024)
 #define SW_MAX_SEQ_LEN ((1 << 20) - 64)  /* every database sequence length <= 1,048,512 */
 
 /* length_threshold value asking the library to choose the inter/intra-task threshold itself

@@ -236,7 +236,7 @@ void main_layouts(const KernelConfig& c, int m, int A1, ProfLayout* lg, ProfLayo
   }
 }
 
-constexpr int kMaxProfileSmem = 220 * 1024;
+constexpr int kMaxProfileSmem = SW_MAX_PROFILE_BYTES;   // include/sw.h
 
 // Workload summary of one regime split (from the sorted, paired layout).
 struct Split {

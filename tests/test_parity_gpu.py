@@ -351,3 +351,63 @@ def test_c5_slice_blosum45_parity():
         ref = _oracle(q, BLOSUM45, 10, 2, db)
         out, _ = _gpu(q, BLOSUM45, 10, 2, db, 3072)
         _assert_equal(out, ref, db, f"C5 slice m={m}")
+
+
+# ------------------------------------------------------------------ north-star invariant and maximum sizes
+def test_query_subject_swap_symmetry():
+    """north_star: "scores are unchanged when query and subject are swapped under a symmetric
+    matrix" (Eq.(1) with w symmetric is symmetric in (q, d): transpose the DP grid, E <-> F).
+    Each database sequence becomes the query of its own search against a one-sequence
+    database holding the original query; both directions go through the CUDA path (group and
+    long regimes) and both equal the oracle."""
+    q = gen.make_query(375)
+    lens = [1, 2, 17, 144, 375, 376, 1500, 3100, 5478]
+    db = _db_from_lengths(lens, seed=41, queries=[q])
+    fwd, _ = _gpu(q, BLOSUM62, 10, 2, db, 1000)
+    _assert_equal(fwd, _oracle(q, BLOSUM62, 10, 2, db), db, "forward")
+    one = gen.Database(q.copy(), np.array([0, q.size], np.int64), np.arange(1))
+    for k in range(db.num_seqs):
+        d = db.residues[db.offsets[k]:db.offsets[k + 1]]
+        for T in (0, 1 << 20):
+            rev, _ = _gpu(d, BLOSUM62, 10, 2, one, T)
+            assert rev[0] == fwd[k], f"seq {k} (len {d.size}) T={T}: swapped {rev[0]} != {fwd[k]}"
+
+
+def test_maximum_query_and_sequence_lengths():
+    """The limits include/sw.h declares: a query of SW_MAX_QUERY_LEN = 65536 residues over a
+    2-letter alphabet (its profile fits SW_MAX_PROFILE_BYTES; many strips; one sequence holds
+    an 8000-residue copy of it, so the s16 pass saturates and the 32-bit recompute decides),
+    the largest protein query the header guarantees (8192), a protein query of 65536 refused
+    with SW_E_UNSUPPORTED, and a database sequence of SW_MAX_SEQ_LEN = 1,048,512 residues in
+    both regimes."""
+    W2 = np.array([[5, -4], [-4, 5]], np.int8)
+    q = (gen.u01(1007, "query", np.arange(1 << 16, dtype=np.uint64)) < 0.5).astype(np.uint8)
+    parts = [(gen.u01(1043 + k, "res", np.arange(n, dtype=np.uint64)) < 0.5).astype(np.uint8)
+             for k, n in enumerate([1, 31, 500, 3100])] + [q[1000:9000]]
+    offs = np.concatenate([[0], np.cumsum([x.size for x in parts])]).astype(np.int64)
+    db = gen.Database(np.concatenate(parts).astype(np.uint8), offs, np.arange(len(parts)))
+    ref = _oracle(q, W2, 10, 2, db)
+    assert ref[-1] == 5 * 8000
+    for T in (0, 3072):
+        out, st = _gpu(q, W2, 10, 2, db, T)
+        _assert_equal(out, ref, db, f"query 65536 (2 letters) T={T}")
+        assert st["recomputed_s32"] >= 1
+
+    q = gen.make_query(8192, seed=9)
+    db = _db_from_lengths([1, 31, 500, 3100, 9000], seed=45, queries=[q])
+    ref = _oracle(q, BLOSUM62, 10, 2, db)
+    for T in (0, 3072):
+        out, _ = _gpu(q, BLOSUM62, 10, 2, db, T)
+        _assert_equal(out, ref, db, f"protein query 8192 T={T}")
+    with pytest.raises(swp.SWError) as e:
+        _gpu(gen.make_query(1 << 16, seed=7), BLOSUM62, 10, 2, db, 3072)
+    assert e.value.status == swp.SW_E_UNSUPPORTED
+
+    q = gen.make_query(144)
+    lmax = (1 << 20) - 64
+    db = _db_from_lengths([lmax, 7, 3073], seed=44)
+    assert db.lengths.max() == lmax
+    ref = _oracle(q, BLOSUM62, 10, 2, db)
+    for T in (0, 1 << 20):
+        out, _ = _gpu(q, BLOSUM62, 10, 2, db, T)
+        _assert_equal(out, ref, db, f"max sequence T={T}")
