@@ -337,7 +337,7 @@ def bench_ours(args, rank, world, local_rank):
     # HOST-resident shard, chunks sorted/packed/uploaded while the previous chunk is searched
     stream_db = None
     if not args.no_stream:
-        chunk = 1 << 25
+        chunk = 1 << 28      # ramps 32M, 64M, 128M, ... (profiles/r01_stream_chunk_sweep.jsonl)
         sw.search_stream(db.residues, db.offsets, T, chunk, queries=qs)      # warm: pinned staging
         t0 = time.perf_counter()
         sw.search_stream(db.residues, db.offsets, T, chunk, queries=qs)

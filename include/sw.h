@@ -126,7 +126,9 @@ int sw_search_batch(sw_handle h, const uint8_t* queries, const int64_t* q_offset
  * background").  A batch of queries (same form as sw_search_batch; queries == NULL: the
  * handle's own query, num_queries/q_offsets ignored) against a HOST-resident database (same
  * CSR form as sw_load_db, only read during the call).  The database is cut into chunks of
- * whole sequences of about chunk_residues residues; each chunk is sorted and packed on the
+ * whole sequences of about chunk_residues residues (the first three ramp up: about 1/8, 1/4
+ * and 1/2 of it, so that the packing of the first chunk, which no search hides, is short);
+ * each chunk is sorted and packed on the
  * host (pinned staging) and copied on an upload stream while the previous chunk is searched,
  * two device slots alternating (kept on the handle for the next call).  The handle's loaded
  * database (if any) is neither used nor changed.

@@ -145,7 +145,7 @@ def sw_search_batch_async(h, queries, d_scores_ptr: int, length_threshold: int, 
                                                    ctypes.c_void_p(stream_ptr)))
 
 
-def sw_search_stream(h, residues, offsets, length_threshold: int = 3072, chunk_residues: int = 1 << 25,
+def sw_search_stream(h, residues, offsets, length_threshold: int = 3072, chunk_residues: int = 1 << 28,
                      queries=None) -> np.ndarray:
     """Search a host-resident database chunk by chunk, uploads overlapped with the search.
     queries=None: the handle's query, returns int32[num_seqs]; else int32[len(queries), num_seqs]."""
@@ -227,7 +227,7 @@ class SmithWaterman:
     def search_batch_into(self, queries, d_scores_ptr: int, length_threshold: int = 3072, stream_ptr: int = 0):
         sw_search_batch_async(self.h, queries, d_scores_ptr, length_threshold, stream_ptr)
 
-    def search_stream(self, residues, offsets, length_threshold: int = 3072, chunk_residues: int = 1 << 25,
+    def search_stream(self, residues, offsets, length_threshold: int = 3072, chunk_residues: int = 1 << 28,
                       queries=None):
         return sw_search_stream(self.h, residues, offsets, length_threshold, chunk_residues, queries)
 

@@ -1086,11 +1086,18 @@ int sw_search_stream(sw_handle h, const uint8_t* queries, const int64_t* q_offse
   std::vector<int64_t> qo(q_offsets, q_offsets + nq + 1);
   SW_CUDA(h, cudaMemcpyAsync(h->d_batch_q, queries, (size_t)qtot, cudaMemcpyHostToDevice, st));
   SW_CUDA(h, cudaStreamSynchronize(st));     // the caller's query buffer is pageable
-  // chunk boundaries: whole sequences, about chunk_residues residues each
+  // chunk boundaries: whole sequences, about chunk_residues residues each; the first three
+  // chunks ramp up (1/8, 1/4, 1/2) because nothing hides the host packing of the first one
+  // (packing runs ~3x faster than the search of the same residues, so doubling stays hidden;
+  // every chunk adds a launch tail, so a longer ramp measured slower:
+  // profiles/r01_stream_chunk_sweep*.jsonl)
+  constexpr int kRamp = 3;
   std::vector<int64_t> cut{0};
   while (cut.back() < num_seqs) {
     const int64_t s0 = cut.back();
-    int64_t e = std::upper_bound(offsets + s0, offsets + num_seqs + 1, offsets[s0] + chunk_residues) - offsets - 1;
+    const int ramp = std::max(0, kRamp - (int)(cut.size() - 1));
+    const int64_t target = std::max<int64_t>(chunk_residues >> ramp, 1);
+    int64_t e = std::upper_bound(offsets + s0, offsets + num_seqs + 1, offsets[s0] + target) - offsets - 1;
     cut.push_back(std::min(std::max(e, s0 + 1), num_seqs));
   }
   const int nchunks = (int)cut.size() - 1;
