@@ -763,9 +763,22 @@ int build_db(sw_handle h, DbState& db, const uint8_t* residues, const int64_t* o
   db.loaded = false;
   std::vector<int64_t> len((size_t)num_seqs);
   for (int64_t k = 0; k < num_seqs; ++k) len[k] = offsets[k + 1] - offsets[k];
+  // stable sort by length descending as a counting sort (lengths <= SW_MAX_SEQ_LEN): linear,
+  // and it sits on the unhidden first chunk of sw_search_stream
   std::vector<int32_t> perm((size_t)num_seqs);
-  std::iota(perm.begin(), perm.end(), 0);
-  std::stable_sort(perm.begin(), perm.end(), [&](int32_t a, int32_t b) { return len[a] > len[b]; });
+  {
+    int64_t lmax = 0;
+    for (int64_t k = 0; k < num_seqs; ++k) lmax = std::max(lmax, len[k]);
+    std::vector<int64_t> start((size_t)lmax + 2, 0);   // start[l] = #sequences longer than l
+    for (int64_t k = 0; k < num_seqs; ++k) ++start[(size_t)len[k]];
+    int64_t acc = 0;
+    for (int64_t l = lmax; l >= 0; --l) {
+      const int64_t c = start[(size_t)l];
+      start[(size_t)l] = acc;
+      acc += c;
+    }
+    for (int64_t k = 0; k < num_seqs; ++k) perm[(size_t)start[(size_t)len[k]]++] = (int32_t)k;
+  }
   db.sorted_len.resize((size_t)num_seqs);
   for (int64_t k = 0; k < num_seqs; ++k) db.sorted_len[k] = len[perm[k]];
   const int n_pairs = (int)((num_seqs + 1) / 2);
