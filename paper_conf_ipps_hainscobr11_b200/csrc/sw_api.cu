@@ -3,6 +3,7 @@
 // stream-ordered launches of the sm_100a kernels.  No CPU fallback: every score is computed
 // by k_search (sw_engine.cuh) on the device.
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <cstdio>
 #include <cstdlib>
@@ -1149,7 +1150,12 @@ int sw_search_stream(sw_handle h, const uint8_t* queries, const int64_t* q_offse
     // host packing + upload of chunk c overlap the device search of chunk c - 1
     // ("copy a slice of the database to the GPU, start aligning, and copy the rest of the
     // database in the background", §VI)
+    const auto tb0 = std::chrono::steady_clock::now();
     rc = build_db(h, ss.db, residues + offsets[s0], off.data(), n, ss.up);
+    if (getenv("SW_DEBUG_STREAM"))
+      fprintf(stderr, "stream chunk %d: %lld seqs, %lld residues, host build+upload %.2f ms\n", c, (long long)n,
+              (long long)(offsets[s1] - offsets[s0]),
+              std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - tb0).count());
     if (rc) break;
     const size_t need = (size_t)nq * (size_t)n * sizeof(int32_t);
     if (ss.d_sc_cap < need) {
