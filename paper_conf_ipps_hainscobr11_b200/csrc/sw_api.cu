@@ -1105,7 +1105,8 @@ int sw_search_stream(sw_handle h, const uint8_t* queries, const int64_t* q_offse
   // (packing runs ~3x faster than the search of the same residues, so doubling stays hidden;
   // every chunk adds a launch tail, so a longer ramp measured slower:
   // profiles/r01_stream_chunk_sweep*.jsonl)
-  constexpr int kRamp = 3;
+  int kRamp = 3;
+  if (const char* f = getenv("SW_STREAM_RAMP")) kRamp = std::max(0, std::min(10, atoi(f)));   // probes
   std::vector<int64_t> cut{0};
   while (cut.back() < num_seqs) {
     const int64_t s0 = cut.back();
