@@ -129,6 +129,10 @@ struct sw_handle_s {
   uint8_t* d_batch_q = nullptr;
   int64_t batch_q_cap = 0;
   cudaEvent_t fork = nullptr;
+  // completion of the last T-mode launch with gangs: the next one waits for it (gang CTAs spin
+  // on each other, so two gang launches must never hold SMs at the same time; sw_engine.cuh
+  // t_gang_item)
+  cudaEvent_t gang_ev = nullptr;
   // stats
   int64_t stat_long = 0, stat_short = 0, stat_launches = 0;
   int stat_nq = 0;
@@ -354,6 +358,14 @@ int ensure_slots(sw_handle h, int n) {
   return SW_OK;
 }
 
+// Make stream st wait for all work the previous call enqueued on the internal slot streams
+// (each slot records `done` after its last query, with its T-mode stream joined back).
+int wait_slots(sw_handle h, cudaStream_t st) {
+  for (QuerySlot& s : h->slots)
+    if (s.stream != st) SW_CUDA(h, cudaStreamWaitEvent(st, s.done, 0));
+  return SW_OK;
+}
+
 int validate_query(sw_handle h, const uint8_t* q, int32_t m) {
   if (!q) return fail(h, SW_E_INVALID, "query is NULL");
   if (m <= 0 || m > SW_MAX_QUERY_LEN) return fail(h, SW_E_INVALID, "query_len out of range [1, 65536]");
@@ -490,8 +502,14 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     rbt = (size_t)pl.grid * nteams * (pl.team_warps + 1) * max_cols_all * sizeof(uint2);
   }
   if (pl.r_passes > 1) {
+    // the recompute list is rare and unknown until the search ran: bound its row buffers by
+    // shrinking the (persistent) recompute grid instead of sizing for every CTA (a database
+    // with a 1M-residue sequence would otherwise need ~15 GB per slot)
     const int nteams = (pl.rcfg.threads / 32) / pl.r_team_warps;
-    rbt = std::max(rbt, (size_t)pl.rgrid * nteams * (pl.r_team_warps + 1) * max_cols_all * sizeof(uint2));
+    const size_t per_cta = (size_t)nteams * (pl.r_team_warps + 1) * max_cols_all * sizeof(uint2);
+    constexpr size_t kRecomputeRbBudget = (size_t)256 << 20;
+    pl.rgrid = (int)std::max<size_t>(1, std::min<size_t>(pl.rgrid, kRecomputeRbBudget / std::max<size_t>(per_cta, 1)));
+    rbt = std::max(rbt, (size_t)pl.rgrid * per_cta);
   }
   rc = grow(h, &s.d_rb_group, &s.rb_group_cap, rbg, "alloc group row buffers", s.stream, true);
   if (rc) return rc;
@@ -503,7 +521,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
   // query stream carries compact letter indices): 21 rows for a 20-letter query instead of 25,
   // so more warps fit in shared memory
   const int a_used = __builtin_popcount(qmask);
-  const int wp_bytes = (int)round_up((int64_t)(a_used + 1) * 32, 128);
+  const int wp_bytes = (int)round_up((int64_t)(a_used + 1) * kWpStride, 128);
   const int per_warp = 2 * (a_used + 1) * 32 * kTmodeC;
   int t_warps = std::min(kTmodeThreads / 32, (kMaxProfileSmem - wp_bytes) / per_warp);
   if (t_warps < 1) use_t = false;
@@ -705,7 +723,9 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     t.rb = s.d_rb_t;
     t.rb_cols = qcols + kPadCols + 1;
     t.hi_mul = 1u << 24;
+    if (t.gang_items > 0) SW_CUDA(h, cudaStreamWaitEvent(s.aux, h->gang_ev, 0));
     SW_CUDA(h, launch_tmode(t, t_grid, t_smem, s.aux));
+    if (t.gang_items > 0) SW_CUDA(h, cudaEventRecord(h->gang_ev, s.aux));
     SW_CUDA(h, cudaEventRecord(s.join, s.aux));
   }
   SW_CUDA(h, launch_search(pl.cfg, p, pl.grid, pl.prof_bytes, st));
@@ -1033,7 +1053,8 @@ int sw_create(sw_handle* out, const uint8_t* query, int32_t query_len, const int
   h->num_sms = prop.multiProcessorCount;
   if (cudaMalloc(&h->d_matrix, (size_t)alphabet_size * alphabet_size) != cudaSuccess ||
       cudaMemcpy(h->d_matrix, matrix, (size_t)alphabet_size * alphabet_size, cudaMemcpyHostToDevice) != cudaSuccess ||
-      cudaEventCreateWithFlags(&h->fork, cudaEventDisableTiming) != cudaSuccess) {
+      cudaEventCreateWithFlags(&h->fork, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&h->gang_ev, cudaEventDisableTiming) != cudaSuccess) {
     sw_destroy(h);
     return SW_E_CUDA;
   }
@@ -1091,6 +1112,8 @@ int sw_search_stream(sw_handle h, const uint8_t* queries, const int64_t* q_offse
   rc = ensure_slots(h, 1);
   if (rc) return rc;
   cudaStream_t st = h->slots[0].stream;
+  rc = wait_slots(h, st);   // earlier calls' slot streams may still read d_batch_q
+  if (rc) return rc;
   const int nq = num_queries;
   const int64_t qtot = q_offsets[nq];
   size_t qcap = (size_t)h->batch_q_cap;
@@ -1227,8 +1250,12 @@ int sw_search_batch_async(sw_handle h, const uint8_t* queries, const int64_t* q_
   }
   cudaStream_t st = reinterpret_cast<cudaStream_t>(cuda_stream);
   const int64_t tot = q_offsets[num_queries];
+  // the previous call's slot streams may still read d_batch_q (its profile builds and query
+  // streams): order the upload after them, whatever stream that call was issued on
+  int rc = wait_slots(h, st);
+  if (rc) return rc;
   size_t cap = (size_t)h->batch_q_cap;
-  int rc = grow(h, &h->d_batch_q, &cap, (size_t)std::max<int64_t>(tot, 1), "alloc batch queries");
+  rc = grow(h, &h->d_batch_q, &cap, (size_t)std::max<int64_t>(tot, 1), "alloc batch queries", st);
   if (rc) return rc;
   h->batch_q_cap = (int64_t)cap;
   if (tot > 0) SW_CUDA(h, cudaMemcpyAsync(h->d_batch_q, queries, (size_t)tot, cudaMemcpyHostToDevice, st));
@@ -1356,6 +1383,7 @@ void sw_destroy(sw_handle h) {
   cudaFree(h->d_tb_dir); cudaFree(h->d_tb_scratch); cudaFree(h->d_tb_result); cudaFree(h->d_tb_ops);
   cudaFree(h->d_tb_query);
   if (h->fork) cudaEventDestroy(h->fork);
+  if (h->gang_ev) cudaEventDestroy(h->gang_ev);
   if (h->h_ovf) cudaFreeHost(h->h_ovf);
   delete h;
 }

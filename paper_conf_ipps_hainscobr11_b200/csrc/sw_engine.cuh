@@ -818,7 +818,7 @@ __device__ __forceinline__ void build_strip_tables(const TParams& p, uint8_t* ta
     dp[r] = pos < ncols ? (uint32_t)cp[pos] : db_pad;
   }
   for (int a = 0; a < A1; ++a) {
-    const int8_t* wrow = wp + a * 32;
+    const int8_t* wrow = wp + a * kWpStride;
 #pragma unroll
     for (int k = 0; k < C / 4; ++k) {
       uint32_t lo = 0, hi = 0;
@@ -1006,8 +1006,14 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const ChainConst
 // gw = rank * gang_warps + warp takes strips gw, gw + GW, ...; the strip hand-off is the team
 // pipeline with its row buffers and progress flags in global memory at gpu scope
 // (release / acquire).  The pair's maximum is combined with atomicMax over the GW warps and
-// emitted by the last one.  (Every gang CTA is resident: the T-mode grid is one wave, and a
-// slot's dependencies were taken by CTAs that started earlier.)
+// emitted by the last one.  Progress needs every rank of a gang to become resident
+// eventually: slots are taken in CTA start order, so the gang slots go to the first
+// gang_items * gang_ctas CTAs that start; a rank that started may spin on a later rank (from
+// the second round of strips on) until that rank's CTA starts.  That CTA waits only for SMs
+// held by kernels that finish on their own: every other CTA of this launch and every group /
+// recompute launch makes progress without waiting on other CTAs, and enqueue_query
+// (sw_api.cu) serialises the T-mode launches that have gangs across the handle's streams, so
+// two gang launches never hold SMs while waiting for each other.
 template <int C>
 __device__ __forceinline__ void t_gang_item(const TParams& p, const ChainConst& c, uint8_t* tab, const int8_t* wp,
                                             int gi, int rank, int warp) {
@@ -1059,11 +1065,13 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   // row; columns = database letters (the database pad letter A maps to the pad value)
   const int A1 = p.A_used + 1;
   const int table_bytes = 2 * A1 * LS;        // lo + hi tables of one warp
-  int8_t* wp = reinterpret_cast<int8_t*>(smem);  // (A_used+1) x 32: w + rho, pad -> -128
-  uint8_t* tables = smem + ((A1 * 32 + 127) & ~127);
+  // (A_used+1) rows of kWpStride bytes: w + rho for database letters d < A, -128 for the
+  // database pad letter d == A (which is 32 for a 32-letter alphabet: the stride must exceed A)
+  int8_t* wp = reinterpret_cast<int8_t*>(smem);
+  uint8_t* tables = smem + ((A1 * kWpStride + 127) & ~127);
   const int warp = threadIdx.x >> 5;
-  for (int t = threadIdx.x; t < A1 * 32; t += blockDim.x) {
-    const int a = t >> 5, d = t & 31;
+  for (int t = threadIdx.x; t < A1 * kWpStride; t += blockDim.x) {
+    const int a = t / kWpStride, d = t % kWpStride;
     int v = kPadValue;
     if (a < p.A_used && d < p.A) v = (int)p.matrix[(int)__fns(p.qmask, 0, a + 1) * p.A + d] + p.rho;
     wp[t] = (int8_t)v;

@@ -104,6 +104,7 @@ KernelConfig recompute_config();
 constexpr int kTmodeC = 16;
 constexpr int kTmodeThreads = 256;
 constexpr int kTmodeMaxQuery = 3072;     // longer queries take team mode for long pairs
+constexpr int kWpStride = 64;            // T-mode substitution table row: database letters 0..A <= 32
 struct TParams {
   const int8_t* matrix;      // A x A, [query][db]
   int A, rho, sigma, max_w, pad_letter;

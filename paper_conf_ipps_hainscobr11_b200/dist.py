@@ -4,7 +4,7 @@ The search shards naturally: every (query, database sequence) score is independe
 ("kernel tasks are independent ... the running time will scale almost linearly with the
 number of GPUs", §IV-B; "pleasantly parallel", L28 §V).  One process per GPU
 loads a shard of the database and searches it with the C ABI; the only collective is one
-gather of the int32 scores (NCCL over NVLink on the B200 box, gloo in the CPU tests).
+gather of the int32 scores to rank 0 (NCCL over NVLink on the B200 box, gloo in the CPU tests).
 
 Partition rule: stable sort of all lengths descending, rank r takes sorted positions
 r, r + G, r + 2G, ... (round-robin).  Every shard then has the same length profile, so both
@@ -29,13 +29,29 @@ def shard_size_bound(n_total: int, world: int) -> int:
     return -(-n_total // world)
 
 
+def assemble(all_idx, blocks, n_total: int):
+    """Scores in global database order from per-rank blocks.
+
+    all_idx: [world, n_pad] global index of every row of every rank's block (-1 = padding);
+    blocks:  [world, nq, n_pad] the ranks' score blocks.  Returns [nq, n_total] (torch)."""
+    import torch
+    world, nq = blocks.shape[0], blocks.shape[1]
+    out = torch.empty((nq, int(n_total)), dtype=blocks.dtype, device=blocks.device)
+    for r in range(world):
+        v = all_idx[r] >= 0
+        out[:, all_idx[r][v]] = blocks[r][:, v]
+    return out
+
+
 class ScoreGather:
-    """Gathers per-rank score blocks [nq, n_local] into rank 0's [nq, n_total] in global order.
+    """Gathers per-rank score blocks [nq, n_local] into [nq, n_total] in global order.
 
     The index map is exchanged once at construction (not on the timed path); each search then
-    costs one all_gather_into_tensor of nq * ceil(N / world) int32 per rank."""
+    costs one collective of nq * ceil(N / world) int32 per rank: a gather to rank 0 (default;
+    only rank 0 holds the world * nq * n_pad receive buffer, 4 GB for C5 with 20 queries) or,
+    with all_gather=True, an all_gather_into_tensor that lands every score on every rank."""
 
-    def __init__(self, global_index, n_total: int, nq: int, group=None, device=None):
+    def __init__(self, global_index, n_total: int, nq: int, group=None, device=None, all_gather: bool = False):
         import torch
         import torch.distributed as dist
 
@@ -43,6 +59,7 @@ class ScoreGather:
         self.group = group
         self.world = dist.get_world_size(group)
         self.rank = dist.get_rank(group)
+        self.all_gather = bool(all_gather)
         self.n_total = int(n_total)
         self.nq = int(nq)
         self.n_pad = shard_size_bound(self.n_total, self.world)
@@ -57,10 +74,13 @@ class ScoreGather:
         dist.all_gather_into_tensor(flat, idx, group=group)   # flat output: gloo and NCCL
         all_idx = flat.view(self.world, self.n_pad)
         self.all_idx = all_idx
-        self.valid = all_idx >= 0
         self.send = torch.zeros((self.nq, self.n_pad), dtype=torch.int32, device=dev)
-        self.recv_flat = torch.empty((self.world * self.nq * self.n_pad,), dtype=torch.int32, device=dev)
-        self.recv = self.recv_flat.view(self.world, self.nq, self.n_pad)
+        self.holds_all = self.all_gather or self.rank == 0
+        if self.holds_all:
+            self.recv_flat = torch.empty((self.world * self.nq * self.n_pad,), dtype=torch.int32, device=dev)
+            self.recv = self.recv_flat.view(self.world, self.nq, self.n_pad)
+        else:
+            self.recv_flat = self.recv = None
 
     def send_ptr(self) -> int:
         """Device pointer of the [nq, n_pad] block the search writes into.  The caller loads
@@ -78,14 +98,18 @@ class ScoreGather:
         return np.concatenate([off, np.full(extra, off[-1], dtype=np.int64)])
 
     def gather(self):
-        """Collective: every rank calls it; returns nothing (the data lands in self.recv)."""
-        self.dist.all_gather_into_tensor(self.recv_flat, self.send.view(-1), group=self.group)
+        """Collective: every rank calls it; returns nothing (the data lands in self.recv on
+        rank 0, or on every rank with all_gather=True)."""
+        if self.all_gather:
+            self.dist.all_gather_into_tensor(self.recv_flat, self.send.view(-1), group=self.group)
+        else:
+            dst = self.dist.get_global_rank(self.group, 0) if self.group is not None else 0
+            glist = list(self.recv.unbind(0)) if self.rank == 0 else None
+            self.dist.gather(self.send, gather_list=glist, dst=dst, group=self.group)
 
     def to_global(self):
-        """[nq, n_total] scores in global database order (valid on every rank after gather)."""
-        import torch
-        out = torch.empty((self.nq, self.n_total), dtype=torch.int32, device=self.recv.device)
-        for r in range(self.world):
-            v = self.valid[r]
-            out[:, self.all_idx[r][v]] = self.recv[r][:, v]
-        return out
+        """[nq, n_total] scores in global database order (after gather(); rank 0, or every
+        rank with all_gather=True)."""
+        if not self.holds_all:
+            raise RuntimeError("to_global() is valid on rank 0 only (gather to rank 0)")
+        return assemble(self.all_idx, self.recv, self.n_total)
