@@ -102,6 +102,17 @@ struct sw_handle_s {
   int num_sms = 0;
   // scoring scheme
   int A = 0, rho = 0, sigma = 0, max_w = 0, min_w = 0;
+  // Kernel-side penalties: any rho, sigma >= 0 is accepted.
+  //  * profile offset c = min(rho, 127 - max_w): the int8 profile holds w + c; delta = rho - c > 0
+  //    selects the WIDE kernels, which add delta back per cell (sw_engine.cuh ChainConstT);
+  //  * s16x2 lanes: rho16 = min(rho, 16384), sigma16 = min(sigma, 16384) and, if either was
+  //    clamped, flag_limit = 16384: for a sequence whose every H is <= flag_limit - 1 a penalty
+  //    above that bound can never make a positive E / F term (E, F <= H - penalty < 0) in either
+  //    system, so its H values are identical; any sequence reaching flag_limit is recomputed;
+  //    rho16 + sigma16 <= 32768 keeps E - sigma, F - sigma >= -32768 (no wrap);
+  //  * s32 lanes (recompute, traceback): the same clamp at 2^29 (every H <= m * 127 < 2^27).
+  int c_prof = 0, rho16 = 0, sigma16 = 0, flag_limit = 0, rho32 = 0, sigma32 = 0;
+  bool wide = false;
   int8_t* d_matrix = nullptr;
   std::vector<uint8_t> query;
   // database (the loaded one; sw_search_stream points db at its chunk slots)
@@ -265,7 +276,7 @@ int make_plan(sw_handle h, int m, const Split& sp, Plan* pl, int force = -1,
   int best_i = -1;
   for (int i = 0; i < menu_size(); ++i) {
     const KernelConfig c = menu_entry(i);
-    if (c.lane != 0) continue;
+    if (c.lane != 0 || (c.wide != 0) != h->wide) continue;
     ProfLayout lg, lt;
     int bytes = 0;
     main_layouts(c, m, A1, &lg, &lt, &bytes);
@@ -300,13 +311,18 @@ int make_plan(sw_handle h, int m, const Split& sp, Plan* pl, int force = -1,
     if (ranked) ranked->emplace_back(cost, i);
     if (cost < best) { best = cost; best_i = i; pl->thr = thr; pl->tail_s = tail_s; pl->thr_full = thr_full; }
   }
-  if (force >= 0 && force < menu_size() && menu_entry(force).lane == 0) best_i = force;
+  // a forced entry must be able to hold the profile values: WIDE entries compute any rho
+  // (delta = 0 included), the others only rho + max_w <= 127
+  auto usable = [&](int i) {
+    return i >= 0 && i < menu_size() && menu_entry(i).lane == 0 && (menu_entry(i).wide || !h->wide);
+  };
+  if (usable(force)) best_i = force;
   pl->cost = best;
   // test hooks: force a menu entry / team size (used by the parity tests to cover every
   // compiled configuration; never needed for correctness)
   if (const char* f = getenv("SW_FORCE_MENU")) {
     const int i = atoi(f);
-    if (i >= 0 && i < menu_size() && menu_entry(i).lane == 0) best_i = i;
+    if (usable(i)) best_i = i;
   }
   if (best_i < 0) return fail(h, SW_E_UNSUPPORTED, "query profile does not fit in shared memory (query_len * (alphabet_size + 1) too large)");
   const KernelConfig c = menu_entry(best_i);
@@ -323,7 +339,7 @@ int make_plan(sw_handle h, int m, const Split& sp, Plan* pl, int force = -1,
     const int w = atoi(f);
     if (w >= 1 && w <= c.threads / 32) pl->team_warps = std::min(w, std::max(1, pl->long_passes));
   }
-  pl->rcfg = recompute_config();
+  pl->rcfg = recompute_config(h->wide);
   pl->rl = make_layout(0, 32, pl->rcfg.Rl, m, A1, 1);
   pl->r_prof_bytes = pl->rl.bytes;
   if (pl->r_prof_bytes > kMaxProfileSmem) return fail(h, SW_E_UNSUPPORTED, "query profile does not fit in shared memory");
@@ -529,7 +545,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
   const int t_smem = wp_bytes + t_warps * per_warp;
   if (use_t) {
     int bps = 0;
-    cudaError_t e = configure_tmode_kernel(t_smem, &bps);
+    cudaError_t e = configure_tmode_kernel(t_smem, &bps, h->wide);
     if (e != cudaSuccess) return cuda_fail(h, e, "configure long-sequence kernel");
     t_grid = std::max(1, bps) * h->num_sms;
     rc = grow(h, &s.d_qpair, &s.qpair_cap, (size_t)(qcols + kPadCols) * sizeof(uint16_t), "alloc query stream",
@@ -543,9 +559,9 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
   cudaStream_t st = s.stream;
   SW_CUDA(h, cudaMemsetAsync(s.d_work, 0, 4 * sizeof(int32_t), st));
   SW_CUDA(h, cudaMemsetAsync(s.d_ovf_count, 0, sizeof(int32_t), st));
-  SW_CUDA(h, launch_profile(s.d_prof, pl.lg, d_q, m, h->d_matrix, h->A, h->rho, st));
-  if (pl.lt.off != pl.lg.off) SW_CUDA(h, launch_profile(s.d_prof, pl.lt, d_q, m, h->d_matrix, h->A, h->rho, st));
-  SW_CUDA(h, launch_profile(s.d_prof + r_off, pl.rl, d_q, m, h->d_matrix, h->A, h->rho, st));
+  SW_CUDA(h, launch_profile(s.d_prof, pl.lg, d_q, m, h->d_matrix, h->A, h->c_prof, st));
+  if (pl.lt.off != pl.lg.off) SW_CUDA(h, launch_profile(s.d_prof, pl.lt, d_q, m, h->d_matrix, h->A, h->c_prof, st));
+  SW_CUDA(h, launch_profile(s.d_prof + r_off, pl.rl, d_q, m, h->d_matrix, h->A, h->c_prof, st));
 
   SearchParams p{};
   p.prof = s.d_prof;
@@ -553,8 +569,10 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
   p.lg = pl.lg;
   p.lt = pl.lt;
   p.pad_letter = h->A;
-  p.rho = h->rho;
-  p.sigma = h->sigma;
+  p.rho = h->rho16;
+  p.sigma = h->sigma16;
+  p.delta = h->rho16 - h->c_prof;
+  p.flag_limit = h->flag_limit;
   p.max_w = h->max_w;
   p.cols = h->db->d_cols;
   p.pair_off = h->db->d_pair_off;
@@ -592,8 +610,10 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     TParams t{};
     t.matrix = h->d_matrix;
     t.A = h->A;
-    t.rho = h->rho;
-    t.sigma = h->sigma;
+    t.rho = h->rho16;
+    t.sigma = h->sigma16;
+    t.delta = h->rho16 - h->c_prof;
+    t.flag_limit = h->flag_limit;
     t.max_w = h->max_w;
     t.pad_letter = h->A;
     t.qmask = qmask;
@@ -738,6 +758,9 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
   r.prof_bytes = pl.r_prof_bytes;
   r.lg = pl.rl;
   r.lt = pl.rl;
+  r.rho = h->rho32;
+  r.sigma = h->sigma32;
+  r.delta = h->rho32 - h->c_prof;
   r.item_list = s.d_ovf_list;
   r.item_count = s.d_ovf_count;
   r.work = s.d_work + 2;
@@ -1041,10 +1064,14 @@ int sw_create(sw_handle* out, const uint8_t* query, int32_t query_len, const int
   }
   int rc = validate_query(h, query, query_len);
   if (rc) { delete h; return rc; }
-  if (gap_open + std::max(h->max_w, 0) > 127 || (int64_t)gap_open + gap_extend > 32000) {
-    delete h;
-    return SW_E_UNSUPPORTED;
-  }
+  h->c_prof = std::min(gap_open, 127 - h->max_w);
+  h->wide = gap_open > h->c_prof;
+  const bool clamp16 = gap_open > 16384 || gap_extend > 16384;
+  h->rho16 = std::min(gap_open, 16384);
+  h->sigma16 = std::min(gap_extend, 16384);
+  h->flag_limit = clamp16 ? std::min(32767 - h->max_w, 16384) : 32767 - h->max_w;
+  h->rho32 = std::min(gap_open, 1 << 29);
+  h->sigma32 = std::min(gap_extend, 1 << 29);
   cudaError_t e = cudaGetDevice(&h->device);
   cudaDeviceProp prop;
   if (e == cudaSuccess) e = cudaGetDeviceProperties(&prop, h->device);
@@ -1333,7 +1360,7 @@ int sw_align(sw_handle h, int64_t seq_index, sw_alignment* out, uint32_t* ops, i
   const int64_t pair = pos >> 1;
   const int half = (int)(pos & 1);
   SW_CUDA(h, launch_traceback(h->d_tb_query, m, h->db->d_cols + h->db->h_pair_off[(size_t)pair], half, (int)n, h->d_matrix,
-                              h->A, h->rho, h->sigma, h->d_tb_dir, h->d_tb_scratch, h->d_tb_result, h->d_tb_ops,
+                              h->A, h->rho32, h->sigma32, h->d_tb_dir, h->d_tb_scratch, h->d_tb_result, h->d_tb_ops,
                               cap_dev, nullptr));
   int res[6];
   SW_CUDA(h, cudaMemcpy(res, h->d_tb_result, sizeof(res), cudaMemcpyDeviceToHost));

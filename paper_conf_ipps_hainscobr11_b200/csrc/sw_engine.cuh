@@ -214,11 +214,18 @@ __device__ __forceinline__ uint32_t subst_row(const uint32_t (&wlo)[(R + 3) / 4]
   }
 }
 
-struct ChainConst {
+// WIDE: rho + max(w) does not fit the int8 profile entry w + rho.  The profile then holds
+// w + c with c = rho - delta (sw_api.cu), and the diagonal term adds delta back on the FMA pipe:
+// t = (hr_up + delta) + (w + c) = H[i-1][j] + w (one more VIADD.16x2 per cell pair).
+template <bool WIDE>
+struct ChainConstT {
+  static constexpr bool kWide = WIDE;
   int rho, sigma;
+  int delta;              // rho - (profile offset c); 0 unless WIDE
   uint32_t padpair;       // residue pair of two pad letters
   uint32_t hi_mul;        // 1 << 24 at run time (SearchParams::hi_mul)
 };
+using ChainConst = ChainConstT<false>;
 
 // The cell update (one row r of one column j, both sequences of the pair).  Besides E, each row
 // keeps t = H[r-1][j] + w(q_r, d_{j+1}) for the NEXT column (the diagonal term of Eq.(1)),
@@ -242,10 +249,11 @@ struct ChainConst {
 // pair and measured 4-5 % slower: issue slots, not the chain, are the tighter limit.)
 // Vertical values enter and leave as (H, F + rho), the format of the lane hand-off and of the
 // strip row buffers.
-template <class L, int R>
+template <class L, int R, bool WIDE = false>
 __device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&t)[R], const uint32_t (&wlo)[(R + 3) / 4],
                                           const uint32_t (&whi)[(R + 3) / 4], uint32_t nrho, uint32_t prho,
-                                          uint32_t nsig, uint32_t& hup, uint32_t& fs, uint32_t& best) {
+                                          uint32_t nsig, uint32_t& hup, uint32_t& fs, uint32_t& best,
+                                          uint32_t dlt = 0u) {
   uint32_t hrup = L::add(hup, nrho), f = L::add(fs, nrho), hprev = 0, h = 0;
 #pragma unroll
   for (int r = 0; r < R; ++r) {
@@ -253,7 +261,8 @@ __device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&t)[R], co
     h = L::hmax(t[r], e[r], f);                                       // H = max(H[i-1][j-1] + w, E, F, 0)
     const uint32_t hr = L::add(h, nrho);                              // H - rho
     e[r] = L::gap(e[r], nsig, hr);                                    // E[j+1] = max(E - sigma, H - rho)
-    t[r] = L::add(hrup, subst_row<L, R>(wlo, whi, r));                // H[i-1][j] + w(q_i, d_{j+1})
+    // H[i-1][j] + w(q_i, d_{j+1}) (WIDE: + delta, the part of rho the int8 profile cannot hold)
+    t[r] = L::add(WIDE ? L::add(hrup, dlt) : hrup, subst_row<L, R>(wlo, whi, r));
     hrup = hr;
     if (r & 1) best = L::max3(best, hprev, h); else hprev = h;
   }
@@ -275,8 +284,8 @@ __device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&t)[R], co
 // ONE_PASS: the query is one strip (no row buffer in or out): the first lane's top input is
 // the constant boundary (0, 0), so the boundary rings and their loads disappear (registers).
 template <class L, int GC, int R, bool TEAM, int PUB = 16, bool GPU_FLAGS = false, int TAG_SHIFT = 20,
-          bool ONE_PASS = false>
-__device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t* prow, int ls, int hi_off,
+          bool ONE_PASS = false, class CC = ChainConst>
+__device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, int ls, int hi_off,
                                              const uint16_t* __restrict__ cols, int ncols,
                                              int half, int steps, int P, int passes_total,
                                              const uint2* __restrict__ rb_in, uint2* __restrict__ rb_out,
@@ -291,6 +300,7 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
   const int gl = lane & (GC - 1);
   const uint32_t nrho = L::splat(-c.rho), prho = L::splat(c.rho);
   const uint32_t nsig = L::splat(-c.sigma);
+  const uint32_t dlt = L::splat(c.delta);
   const int hshift = 8 * half;
   constexpr int CB = chunk_bytes<R>();
   const bool store_out = !ONE_PASS && (gl == GC - 1) && (P < passes_total - 1);
@@ -368,7 +378,7 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
       load_prof<R, CB, GC * CB>(wlo, prow + alo * ls);
     }
     uint32_t hup = x_hr, fs = x_f;
-    cell_rows<L, R>(e, t, wlo, whi, nrho, prho, nsig, hup, fs, best);
+    cell_rows<L, R, CC::kWide>(e, t, wlo, whi, nrho, prho, nsig, hup, fs, best, dlt);
     y_hr = hup; y_f = fs; y_res = x_res;
     // last lane: save the strip's bottom row for the next strip (not after the last strip);
     // fill steps write neutral values (index -1 keeps its neutral entry) that the real column
@@ -417,7 +427,7 @@ __device__ __forceinline__ uint32_t run_pass(const ChainConst& c, const uint8_t*
 template <class L>
 __device__ __forceinline__ void emit(const SearchParams& p, uint32_t b, int pair, int half) {
   if constexpr (L::kSeqs == 2) {
-    const int limit = 32767 - p.max_w;
+    const int limit = p.flag_limit;
     const int s0 = 2 * pair, s1 = 2 * pair + 1;
     const int lo = (int)(int16_t)(b & 0xffffu), hi = (int)(int16_t)(b >> 16);
     if (lo >= limit) p.ovf_list[atomicAdd(p.ovf_count, 1)] = s0; else p.scores[p.perm[s0]] = lo;
@@ -469,8 +479,8 @@ struct GsState {
 // MULTI = false: the query fits one strip (p.short_passes == 1), so there is no strip row
 // buffer: the first lane's top input is the constant boundary (H, F + rho) = (0, 0) and only
 // the residues go through the fetch ring (8 registers and 2 selects per step fewer).
-template <class L, int R, bool MULTI>
-__device__ __forceinline__ void group_stream(const SearchParams& p, const ChainConst& c, const uint8_t* pbase,
+template <class L, int R, bool MULTI, class CC>
+__device__ __forceinline__ void group_stream(const SearchParams& p, const CC& c, const uint8_t* pbase,
                                              uint2* __restrict__ rb, volatile GsState* gs) {
   static_assert(R % 4 == 0 || R >= 12, "R < 12 must be a multiple of 4");
   constexpr int kGap = 4;
@@ -478,6 +488,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
   const uint32_t not0 = lane == 0 ? 0u : 1u;
   const uint32_t nrho = L::splat(-c.rho), prho = L::splat(c.rho);
   const uint32_t nsig = L::splat(-c.sigma);
+  const uint32_t dlt = L::splat(c.delta);
   constexpr int CB = chunk_bytes<R>();
   constexpr int kStripBytes = chunks_per_lane<R>() * 32 * CB;   // chunks x 32 lanes x CB bytes
   constexpr int kEndLen = 0xffffff;            // the END segment (after the last pair) never ends
@@ -602,7 +613,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
     }
     fetch(K);
     uint32_t hup = x_hr, fs = x_f;
-    cell_rows<L, R>(e, t, wlo, whi, nrho, prho, nsig, hup, fs, best);
+    cell_rows<L, R, CC::kWide>(e, t, wlo, whi, nrho, prho, nsig, hup, fs, best, dlt);
     y_hr = hup; y_f = fs; y_res = x_res;
     // keep the next step's residue shuffle (and so its profile loads) after this step's rows:
     // hoisting them would keep a second set of profile words live
@@ -646,7 +657,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const ChainC
   }
 }
 
-template <class L, int G, int Rs, int Rl, int NT>
+template <class L, int G, int Rs, int Rl, int NT, bool WIDE = false>
 __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
   constexpr int kWarps = NT / 32;
   extern __shared__ __align__(128) uint8_t smem[];
@@ -675,9 +686,10 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
   }
   mbar_wait(&mbar, 0);
 
-  ChainConst c;
+  ChainConstT<WIDE> c;
   c.rho = p.rho;
   c.sigma = p.sigma;
+  c.delta = p.delta;
   c.padpair = (uint32_t)p.pad_letter | ((uint32_t)p.pad_letter << 8);
   c.hi_mul = p.hi_mul;
 
@@ -839,7 +851,7 @@ __device__ __forceinline__ void build_strip_tables(const TParams& p, uint8_t* ta
 
 // scores of long pair `item` from its reduced s16x2 maximum (or its overflow flags)
 __device__ __forceinline__ void emit_t(const TParams& p, uint32_t bb, int item) {
-  const int limit = 32767 - p.max_w;
+  const int limit = p.flag_limit;
   const int s0 = 2 * item, s1 = 2 * item + 1;
   const int lo = (int)(int16_t)(bb & 0xffffu), hi = (int)(int16_t)(bb >> 16);
   if (lo >= limit) p.ovf_list[atomicAdd(p.ovf_count, 1)] = s0; else p.scores[p.perm[s0]] = lo;
@@ -853,8 +865,8 @@ __device__ __forceinline__ void emit_t(const TParams& p, uint32_t bb, int item) 
 // with at least this many strips (fewer: the item is parked in *parked and the loop returns,
 // so that the CTA can regroup into smaller teams for the remaining, shorter items).  Items
 // [0, gang_items) belong to the gangs (t_gang_item); the queue starts after them.
-template <int C>
-__device__ __forceinline__ void t_team_loop(const TParams& p, const ChainConst& c, uint8_t* tab,
+template <int C, class CC>
+__device__ __forceinline__ void t_team_loop(const TParams& p, const CC& c, uint8_t* tab,
                                             const int8_t* wp, int W, int team, int wt, int first_item,
                                             int min_strips, int* parked, uint32_t* prog, uint2* rb,
                                             int32_t* sitem, uint32_t* sred) {
@@ -918,8 +930,8 @@ struct TStream {
   int item[kTQ], base[kTQ], S[kTQ], rem[kTQ], mlo[kTQ], mhi[kTQ];
 };
 
-template <int C>
-__device__ __forceinline__ void t_team_stream(const TParams& p, const ChainConst& c, uint8_t* tab,
+template <int C, class CC>
+__device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uint8_t* tab,
                                               const int8_t* wp, int W, int team, int wt, int first_item,
                                               uint32_t* prog, uint2* rb, TStream* ts) {
   using L = LaneS16x2;
@@ -1014,8 +1026,8 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const ChainConst
 // recompute launch makes progress without waiting on other CTAs, and enqueue_query
 // (sw_api.cu) serialises the T-mode launches that have gangs across the handle's streams, so
 // two gang launches never hold SMs while waiting for each other.
-template <int C>
-__device__ __forceinline__ void t_gang_item(const TParams& p, const ChainConst& c, uint8_t* tab, const int8_t* wp,
+template <int C, class CC>
+__device__ __forceinline__ void t_gang_item(const TParams& p, const CC& c, uint8_t* tab, const int8_t* wp,
                                             int gi, int rank, int warp) {
   using L = LaneS16x2;
   constexpr int CB = chunk_bytes<C>();
@@ -1052,7 +1064,7 @@ __device__ __forceinline__ void t_gang_item(const TParams& p, const ChainConst& 
   }
 }
 
-template <int C, int NT>
+template <int C, int NT, bool WIDE = false>
 __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   constexpr int kWarps = NT / 32;
   constexpr int LS = 32 * C;
@@ -1073,15 +1085,16 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   for (int t = threadIdx.x; t < A1 * kWpStride; t += blockDim.x) {
     const int a = t / kWpStride, d = t % kWpStride;
     int v = kPadValue;
-    if (a < p.A_used && d < p.A) v = (int)p.matrix[(int)__fns(p.qmask, 0, a + 1) * p.A + d] + p.rho;
+    if (a < p.A_used && d < p.A) v = (int)p.matrix[(int)__fns(p.qmask, 0, a + 1) * p.A + d] + p.rho - p.delta;
     wp[t] = (int8_t)v;
   }
   if (threadIdx.x == 0) sparked = -1;
   __syncthreads();
   if (warp >= p.warps) return;
-  ChainConst c;
+  ChainConstT<WIDE> c;
   c.rho = p.rho;
   c.sigma = p.sigma;
+  c.delta = p.delta;
   c.padpair = (uint32_t)p.A_used * 0x101u;     // the query stream's (compact) pad letter
   c.hi_mul = p.hi_mul;
   uint8_t* tab = tables + warp * table_bytes;
@@ -1117,32 +1130,32 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
                    rb_cta + (int64_t)team * (W + 1) * p.rb_cols, &sts[team]);
 }
 
-template <int C, int NT>
+template <int C, int NT, bool WIDE>
 cudaError_t launch_search_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st) {
-  k_search_t<C, NT><<<grid, NT, smem_bytes, st>>>(p);
+  k_search_t<C, NT, WIDE><<<grid, NT, smem_bytes, st>>>(p);
   return cudaGetLastError();
 }
 
-template <int C, int NT>
+template <int C, int NT, bool WIDE>
 cudaError_t configure_tmode(int smem_bytes, int* blocks_per_sm) {
   cudaError_t e =
-      cudaFuncSetAttribute(k_search_t<C, NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+      cudaFuncSetAttribute(k_search_t<C, NT, WIDE>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search_t<C, NT>, NT, smem_bytes);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search_t<C, NT, WIDE>, NT, smem_bytes);
 }
 
-template <class L, int G, int Rs, int Rl, int NT>
+template <class L, int G, int Rs, int Rl, int NT, bool WIDE>
 cudaError_t launch_search_t(const SearchParams& p, int grid, int smem_bytes, cudaStream_t st) {
-  k_search<L, G, Rs, Rl, NT><<<grid, NT, smem_bytes, st>>>(p);
+  k_search<L, G, Rs, Rl, NT, WIDE><<<grid, NT, smem_bytes, st>>>(p);
   return cudaGetLastError();
 }
 
-template <class L, int G, int Rs, int Rl, int NT>
+template <class L, int G, int Rs, int Rl, int NT, bool WIDE>
 cudaError_t configure_t(int smem_bytes, int* blocks_per_sm) {
-  cudaError_t e = cudaFuncSetAttribute(k_search<L, G, Rs, Rl, NT>,
+  cudaError_t e = cudaFuncSetAttribute(k_search<L, G, Rs, Rl, NT, WIDE>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search<L, G, Rs, Rl, NT>, NT,
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search<L, G, Rs, Rl, NT, WIDE>, NT,
                                                        smem_bytes);
 }
 

@@ -40,13 +40,15 @@ struct ProfLayout {
 
 // One persistent search launch for one query.
 struct SearchParams {
-  // query profile (w(q_i, a) + rho as int8, -128 for pad letters / rows), staged as one blob
+  // query profile (w(q_i, a) + rho - delta as int8, -128 for pad letters / rows), staged as one blob
   const uint8_t* prof;       // global blob: group image then (if different) team image
   int prof_bytes;            // blob size (multiple of 16)
   ProfLayout lg;             // group-mode image
   ProfLayout lt;             // team-mode image (may alias lg)
   int pad_letter;            // == A
-  int rho, sigma, max_w;
+  int rho, sigma, max_w;     // rho, sigma: the kernel's (clamped) penalties, DESIGN.md "Integer widths"
+  int delta;                 // rho - profile offset (> 0 only for WIDE kernels)
+  int flag_limit;            // s16x2: a best >= flag_limit is recomputed in 32 bits
   // database, sorted by length descending and paired (2p, 2p+1)
   const uint16_t* cols;      // interleaved columns: cols[pair_off[p] + j] = d_lo[j] | d_hi[j] << 8
   const int64_t* pair_off;   // in u16 units
@@ -87,6 +89,7 @@ struct KernelConfig {
   int Rs;
   int Rl;
   int threads;   // CTA size (fewer threads for the register-heavy entries)
+  int wide;      // 1: rho + max(w) > 127 variant (ChainConstT<true>, sw_engine.cuh)
 };
 
 // Launch one search; returns the CUDA error of the launch.
@@ -97,7 +100,7 @@ cudaError_t configure_kernel(const KernelConfig& cfg, int smem_bytes, int* block
 // The menu of compiled configurations.
 int menu_size();
 KernelConfig menu_entry(int i);
-KernelConfig recompute_config();
+KernelConfig recompute_config(bool wide);
 
 // T-mode (transposed long-sequence kernel, sw_engine.cuh k_search_t): C database positions
 // per lane, one CTA team of up to kTmodeThreads / 32 warps per long pair.
@@ -108,6 +111,7 @@ constexpr int kWpStride = 64;            // T-mode substitution table row: datab
 struct TParams {
   const int8_t* matrix;      // A x A, [query][db]
   int A, rho, sigma, max_w, pad_letter;
+  int delta, flag_limit;     // as SearchParams (the strip tables hold w + rho - delta)
   const uint16_t* qpair;     // query as (q | q << 8), qcols + kPadCols entries, pad beyond m
   int qcols;                 // query length rounded up to 8
   const uint16_t* cols;
@@ -138,7 +142,7 @@ struct TParams {
 };
 
 cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st);
-cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm);
+cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm, bool wide);
 cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, uint32_t qmask, cudaStream_t st);
 
 // Traceback of one pair (sw_traceback.cu): dir = m*n bytes, scratch = 7*m ints, result = 6 ints.
@@ -146,7 +150,8 @@ cudaError_t launch_traceback(const uint8_t* q, int m, const uint16_t* dcols, int
                              int rho, int sigma, uint8_t* dir, int* scratch, int* result, uint32_t* ops, int ops_cap,
                              cudaStream_t st);
 
-// Profile image build: byte(rep, a, i) = (i < m && a < A) ? W[q_i][a] + rho : -128.
+// Profile image build: byte(rep, a, i) = (i < m && a < A) ? W[q_i][a] + rho : -128 (rho here is the
+// profile offset c = rho - delta).
 cudaError_t launch_profile(uint8_t* blob, const ProfLayout& L, const uint8_t* q, int m, const int8_t* W, int A,
                            int rho, cudaStream_t st);
 

@@ -22,11 +22,13 @@ cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, uint32_t
 }
 
 cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st) {
-  return launch_search_tmode<kTmodeC, kTmodeThreads>(p, grid, smem_bytes, st);
+  if (p.delta > 0) return launch_search_tmode<kTmodeC, kTmodeThreads, true>(p, grid, smem_bytes, st);
+  return launch_search_tmode<kTmodeC, kTmodeThreads, false>(p, grid, smem_bytes, st);
 }
 
-cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm) {
-  return configure_tmode<kTmodeC, kTmodeThreads>(smem_bytes, blocks_per_sm);
+cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm, bool wide) {
+  if (wide) return configure_tmode<kTmodeC, kTmodeThreads, true>(smem_bytes, blocks_per_sm);
+  return configure_tmode<kTmodeC, kTmodeThreads, false>(smem_bytes, blocks_per_sm);
 }
 
 }  // namespace swb
