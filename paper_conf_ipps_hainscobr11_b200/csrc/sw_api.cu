@@ -458,10 +458,27 @@ int64_t choose_threshold(sw_handle h, int m) {
   return chosen;
 }
 
+// Long-query mode: the smallest query-profile image (the s32 recompute's team image, 32 lanes x
+// 16 rows per strip, one replica; every group / team image is at least as large) exceeds the
+// shared memory of one CTA.  SW_LONG_QUERY=1 forces the mode (tests, probes).
+bool long_query_mode(sw_handle h, int m) {
+  if (const char* f = getenv("SW_LONG_QUERY"))
+    if (f[0] == '1') return true;
+  const KernelConfig rc = recompute_config(h->wide);
+  return make_layout(0, 32, rc.Rl, m, h->A + 1, 1).bytes > kMaxProfileSmem;
+}
+
 // Enqueue one query (device query pointer) on slot s; scores to d_out (device, caller order).
 int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t qmask, int32_t* d_out, int32_t T,
                   int32_t* h_ovf, cudaEvent_t* ev) {
-  if (T == SW_AUTO_THRESHOLD) T = (int32_t)std::min<int64_t>(choose_threshold(h, m), INT32_MAX);
+  // Long-query mode: when even the smallest query-profile image
+  // does not fit one CTA's shared memory, every pair takes T-mode, which streams the query
+  // from global memory and builds its substitution tables per database strip (no query
+  // profile), and the flagged sequences are recomputed by T-mode's 32-bit instantiation.
+  // The threshold then only names the path: every sequence is a "long" one.
+  const bool longq = long_query_mode(h, m);
+  if (longq) T = 0;
+  else if (T == SW_AUTO_THRESHOLD) T = (int32_t)std::min<int64_t>(choose_threshold(h, m), INT32_MAX);
   h->last_threshold = T;
   int64_t n_long_seqs = 0;
   const Split sp = make_split(h, T, &n_long_seqs);
@@ -472,8 +489,8 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     const auto it = h->tuned.find({m, T});
     if (it != h->tuned.end()) force = it->second;
   }
-  Plan pl;
-  int rc = make_plan(h, m, sp, &pl, force);
+  Plan pl{};
+  int rc = longq ? SW_OK : make_plan(h, m, sp, &pl, force);
   if (rc) return rc;
   // Long pairs: T-mode (strips along the database sequence) when the query is short enough
   // that team mode would have few query strips to spread over warps; team mode otherwise.
@@ -485,9 +502,8 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     if (!strcmp(f, "team")) use_t = false;
     if (!strcmp(f, "t")) use_t = n_long > 0;
   }
-  // T-mode progress tags hold the query column in 13 bits (sw_engine.cuh t_team_stream)
-  if (round_up(m, 8) + kPadCols + 36 >= 8192) use_t = false;
-  if (use_t) {
+  if (longq) use_t = n_long > 0;
+  if (use_t && !longq) {
     // the main launch then only sees the short pairs: plan it for them
     Split ss = sp;
     ss.n_long = 0; ss.long_cols = 0; ss.long_max_cols = 0;
@@ -559,9 +575,11 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
   cudaStream_t st = s.stream;
   SW_CUDA(h, cudaMemsetAsync(s.d_work, 0, 4 * sizeof(int32_t), st));
   SW_CUDA(h, cudaMemsetAsync(s.d_ovf_count, 0, sizeof(int32_t), st));
-  SW_CUDA(h, launch_profile(s.d_prof, pl.lg, d_q, m, h->d_matrix, h->A, h->c_prof, st));
-  if (pl.lt.off != pl.lg.off) SW_CUDA(h, launch_profile(s.d_prof, pl.lt, d_q, m, h->d_matrix, h->A, h->c_prof, st));
-  SW_CUDA(h, launch_profile(s.d_prof + r_off, pl.rl, d_q, m, h->d_matrix, h->A, h->c_prof, st));
+  if (!longq) {
+    SW_CUDA(h, launch_profile(s.d_prof, pl.lg, d_q, m, h->d_matrix, h->A, h->c_prof, st));
+    if (pl.lt.off != pl.lg.off) SW_CUDA(h, launch_profile(s.d_prof, pl.lt, d_q, m, h->d_matrix, h->A, h->c_prof, st));
+    SW_CUDA(h, launch_profile(s.d_prof + r_off, pl.rl, d_q, m, h->d_matrix, h->A, h->c_prof, st));
+  }
 
   SearchParams p{};
   p.prof = s.d_prof;
@@ -604,9 +622,13 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     // T-mode runs on the slot's second stream, concurrently with the group launch: its CTAs
     // take every SM first (launched first), and as they run out of long pairs the group
     // launch's CTAs take their SMs, so the longest long pair overlaps the short-pair work.
+    // (long-query mode: T-mode is the only search launch and runs on the slot's stream)
     SW_CUDA(h, launch_qpair(s.d_qpair, d_q, m, qcols + kPadCols, qmask, st));
-    SW_CUDA(h, cudaEventRecord(s.fork, st));
-    SW_CUDA(h, cudaStreamWaitEvent(s.aux, s.fork, 0));
+    cudaStream_t tst = longq ? st : s.aux;
+    if (!longq) {
+      SW_CUDA(h, cudaEventRecord(s.fork, st));
+      SW_CUDA(h, cudaStreamWaitEvent(s.aux, s.fork, 0));
+    }
     TParams t{};
     t.matrix = h->d_matrix;
     t.A = h->A;
@@ -728,12 +750,12 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     if (t.gang_items > 0) {
       const int GW = t.gang_ctas * t.gang_warps;
       const size_t ints = 1 + 3 * (size_t)t.gang_items + (size_t)t.gang_items * (GW + 1);
-      rc = grow(h, &s.d_gang, &s.gang_cap, ints * sizeof(int32_t), "alloc gang scratch", s.aux);
+      rc = grow(h, &s.d_gang, &s.gang_cap, ints * sizeof(int32_t), "alloc gang scratch", tst);
       if (rc) return rc;
       rc = grow(h, &s.d_grb, &s.grb_cap, (size_t)t.gang_items * (GW + 1) * (qcols + kPadCols + 1) * sizeof(uint2),
-                "alloc gang row buffers", s.aux, true);
+                "alloc gang row buffers", tst, true);
       if (rc) return rc;
-      SW_CUDA(h, cudaMemsetAsync(s.d_gang, 0, ints * sizeof(int32_t), s.aux));
+      SW_CUDA(h, cudaMemsetAsync(s.d_gang, 0, ints * sizeof(int32_t), tst));
       t.gang_ctr = s.d_gang;
       t.gbest = s.d_gang + 1;
       t.gdone = s.d_gang + 1 + 2 * t.gang_items;
@@ -743,10 +765,42 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     t.rb = s.d_rb_t;
     t.rb_cols = qcols + kPadCols + 1;
     t.hi_mul = 1u << 24;
-    if (t.gang_items > 0) SW_CUDA(h, cudaStreamWaitEvent(s.aux, h->gang_ev, 0));
-    SW_CUDA(h, launch_tmode(t, t_grid, t_smem, s.aux));
-    if (t.gang_items > 0) SW_CUDA(h, cudaEventRecord(h->gang_ev, s.aux));
+    if (t.gang_items > 0) SW_CUDA(h, cudaStreamWaitEvent(tst, h->gang_ev, 0));
+    SW_CUDA(h, launch_tmode(t, t_grid, t_smem, tst));
+    if (t.gang_items > 0) SW_CUDA(h, cudaEventRecord(h->gang_ev, tst));
+    if (longq) {
+      SW_CUDA(h, cudaEventRecord(ev[1], st));
+      // exact 32-bit recompute of the flagged sequences: T-mode's LaneS32 instantiation (one
+      // sequence per strip table; items from the overflow list, exits at once when it is empty)
+      TParams r = t;
+      r.rho = h->rho32;
+      r.sigma = h->sigma32;
+      r.delta = h->rho32 - h->c_prof;
+      r.item_list = s.d_ovf_list;
+      r.item_count = s.d_ovf_count;
+      r.work = s.d_work + 2;
+      r.gang_items = 0;
+      r.big_strips = 1 << 30;
+      r.team_warps = std::min(2, t.warps);
+      while (t.warps % r.team_warps) --r.team_warps;
+      const int smem32 = wp_bytes + t.warps * per_warp / 2;
+      int bps = 0;
+      cudaError_t e = configure_tmode_kernel(smem32, &bps, h->wide, true);
+      if (e != cudaSuccess) return cuda_fail(h, e, "configure long-sequence recompute kernel");
+      SW_CUDA(h, launch_tmode(r, std::min(t_grid, std::max(1, bps) * h->num_sms), smem32, st, true));
+      SW_CUDA(h, cudaEventRecord(ev[2], st));
+      SW_CUDA(h, cudaMemcpyAsync(h_ovf, s.d_ovf_count, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+      h->stat_long += n_long_seqs;
+      h->stat_short += h->db->n_seqs - n_long_seqs;
+      h->stat_launches += 6;
+      return SW_OK;
+    }
     SW_CUDA(h, cudaEventRecord(s.join, s.aux));
+  } else if (longq) {   // no sequences: nothing to search
+    SW_CUDA(h, cudaEventRecord(ev[1], st));
+    SW_CUDA(h, cudaEventRecord(ev[2], st));
+    SW_CUDA(h, cudaMemcpyAsync(h_ovf, s.d_ovf_count, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+    return SW_OK;
   }
   SW_CUDA(h, launch_search(pl.cfg, p, pl.grid, pl.prof_bytes, st));
   if (use_t) SW_CUDA(h, cudaStreamWaitEvent(st, s.join, 0));
@@ -933,7 +987,7 @@ int autotune(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq,
   const double residues = std::accumulate(h->db->sorted_len.begin(), h->db->sorted_len.end(), 0.0);
   for (int k = 0; k < nq; ++k) {
     const int m = (int)(qoff[k + 1] - qoff[k]);
-    if ((double)m * residues < kTuneMinCells) continue;
+    if ((double)m * residues < kTuneMinCells || long_query_mode(h, m)) continue;
     int32_t Tk = T;
     if (Tk == SW_AUTO_THRESHOLD) Tk = (int32_t)std::min<int64_t>(choose_threshold(h, m), INT32_MAX);
     const std::pair<int, int32_t> key{m, Tk};

@@ -141,6 +141,15 @@ __device__ __forceinline__ uint32_t ld_acquire_smem(const uint32_t* p) {
 __device__ __forceinline__ void st_release_smem(uint32_t* p, uint32_t v) {
   asm volatile("st.release.cta.shared::cta.u32 [%0], %1;" ::"r"(smem_u32(p)), "r"(v) : "memory");
 }
+// 64-bit progress tags (T-mode team stream: running strip index << 32 | query columns done)
+__device__ __forceinline__ unsigned long long ld_acquire_smem(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.cta.shared::cta.u64 %0, [%1];" : "=l"(v) : "r"(smem_u32(p)) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_smem(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.release.cta.shared::cta.u64 [%0], %1;" ::"r"(smem_u32(p)), "l"(v) : "memory");
+}
 // gpu-scope flags in global memory (T-mode gangs: a strip pipeline across CTAs)
 __device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
   uint32_t v;
@@ -284,17 +293,19 @@ __device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&t)[R], co
 // ONE_PASS: the query is one strip (no row buffer in or out): the first lane's top input is
 // the constant boundary (0, 0), so the boundary rings and their loads disappear (registers).
 template <class L, int GC, int R, bool TEAM, int PUB = 16, bool GPU_FLAGS = false, int TAG_SHIFT = 20,
-          bool ONE_PASS = false, class CC = ChainConst>
+          bool ONE_PASS = false, class CC = ChainConst, class TagT = uint32_t>
 __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, int ls, int hi_off,
                                              const uint16_t* __restrict__ cols, int ncols,
                                              int half, int steps, int P, int passes_total,
                                              const uint2* __restrict__ rb_in, uint2* __restrict__ rb_out,
-                                             const uint32_t* prog_in, uint32_t* prog_out, uint32_t best,
+                                             const TagT* prog_in, TagT* prog_out, uint32_t best,
                                              int tagP = -1) {
   // progress tags: (strip index << TAG_SHIFT) | columns done, monotonic per flag slot; the
-  // strip index is the pass P, or the team stream's running strip index tagP
-  const uint32_t tag_base = (uint32_t)(tagP >= 0 ? tagP : P) << TAG_SHIFT;
-  const uint32_t tag_prev = tag_base - (1u << TAG_SHIFT);
+  // strip index is the pass P, or the team stream's running strip index tagP (64-bit tags,
+  // TAG_SHIFT = 32: the running index is unbounded and the query may have up to 2^20 columns)
+  static_assert(TAG_SHIFT < 8 * (int)sizeof(TagT), "tag type too narrow");
+  const TagT tag_base = (TagT)(tagP >= 0 ? tagP : P) << TAG_SHIFT;
+  const TagT tag_prev = tag_base - ((TagT)1 << TAG_SHIFT);
   static_assert(R % 4 == 0 || R >= 12, "R < 12 must be a multiple of 4");
   const int lane = threadIdx.x & 31;
   const int gl = lane & (GC - 1);
@@ -328,7 +339,7 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
   uint32_t rrA[4], rhA[4], rfA[4], rrB[4], rhB[4], rfB[4];
 #pragma unroll
   for (int k = 0; k < 4; ++k) { rhA[k] = rfA[k] = rhB[k] = rfB[k] = 0; rrA[k] = rrB[k] = c.padpair; }
-  uint32_t known = 0;   // team mode: last progress value seen for strip P - 1
+  TagT known = 0;       // team mode: last progress value seen for strip P - 1
   // Every lane of the chain runs the fetch (same addresses as its lane 0: broadcast loads, no
   // extra traffic) so the warp never diverges; only lane 0 consumes the values.  One fetch per
   // group of 4 steps (lane-0 columns c0 .. c0 + 3), one team-mode wait per group: a
@@ -339,9 +350,10 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
     for (int k = 0; k < 4; ++k) rr[k] = cols[min(c0 + k + 1, cmax)];
     if (from_prev) {
       if constexpr (TEAM) {
-        const uint32_t need = tag_prev | (uint32_t)(min(c0 + 3, rlast) + 1);
+        const TagT need = tag_prev | (TagT)(min(c0 + 3, rlast) + 1);
         while (known < need) {
-          known = GPU_FLAGS ? ld_acquire_gpu(prog_in) : ld_acquire_smem(prog_in);
+          if constexpr (GPU_FLAGS) known = ld_acquire_gpu(prog_in);
+          else known = ld_acquire_smem(prog_in);
           if (known < need) __nanosleep(32);
         }
       }
@@ -396,8 +408,8 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
       const int done = col;   // the last lane's columns < col are stored
       if (done > 0 && (PUB == 4 || (done & 15) < 4 || done > rlast))
       {
-        if constexpr (GPU_FLAGS) st_release_gpu(prog_out, tag_base | (uint32_t)min(done, rlast + 1));
-        else st_release_smem(prog_out, tag_base | (uint32_t)min(done, rlast + 1));
+        if constexpr (GPU_FLAGS) st_release_gpu(prog_out, tag_base | (TagT)min(done, rlast + 1));
+        else st_release_smem(prog_out, tag_base | (TagT)min(done, rlast + 1));
       }
     }
   };
@@ -778,13 +790,13 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
         constexpr int CBs = chunk_bytes<Rs>();
         const uint8_t* prow = smem + p.lg.off + gi * p.lg.rs + gl * CBs;
         b = run_pass<L, G, Rs, false, 16, false, 20, true>(c, prow, p.lg.ls, 0, cp, ncols, 0, steps, 0, 1, rb + 1,
-                                                            rb + 1, nullptr, nullptr, b);
+                                                            rb + 1, (uint32_t*)nullptr, (uint32_t*)nullptr, b);
       } else {
         for (int P = 0; P < p.short_passes; ++P) {
           constexpr int CBs = chunk_bytes<Rs>();
           const uint8_t* prow = smem + p.lg.off + gi * p.lg.rs + (P * chunks_per_lane<Rs>() * G + gl) * CBs;
           b = run_pass<L, G, Rs, false>(c, prow, p.lg.ls, 0, cp, ncols, 0, steps, P, p.short_passes, rb + 1, rb + 1,
-                                        nullptr, nullptr, b);
+                                        (uint32_t*)nullptr, (uint32_t*)nullptr, b);
           __syncwarp();   // strip P's bottom row (written by lane G-1) is read by lane 0 in strip P+1
         }
       }
@@ -814,9 +826,10 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
 // Build warp's strip tables for strip P of a long pair: position pos = P*LS + lane*C + r;
 // P_lo[a][pos] = w(a, d_lo[pos]) + rho (a = compact query letter), P_hi likewise, chunk-major
 // and lane-private like the query profile (every lane writes and later reads only its chunks).
-template <int C>
+// SEQS = 1 (32-bit recompute of one flagged sequence): only P_lo, for the pair's half-th sequence.
+template <int C, int SEQS = 2>
 __device__ __forceinline__ void build_strip_tables(const TParams& p, uint8_t* tab, const int8_t* wp,
-                                                   const uint16_t* cp, int ncols, int P) {
+                                                   const uint16_t* cp, int ncols, int P, int half = 0) {
   constexpr int CB = chunk_bytes<C>();
   constexpr int LS = 32 * C;
   const int lane = threadIdx.x & 31;
@@ -837,13 +850,17 @@ __device__ __forceinline__ void build_strip_tables(const TParams& p, uint8_t* ta
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
         const uint32_t d = dp[4 * k + j];
-        lo |= (uint32_t)(uint8_t)wrow[d & 0xff] << (8 * j);
-        hi |= (uint32_t)(uint8_t)wrow[d >> 8] << (8 * j);
+        if constexpr (SEQS == 2) {
+          lo |= (uint32_t)(uint8_t)wrow[d & 0xff] << (8 * j);
+          hi |= (uint32_t)(uint8_t)wrow[d >> 8] << (8 * j);
+        } else {
+          lo |= (uint32_t)(uint8_t)wrow[(d >> (8 * half)) & 0xff] << (8 * j);
+        }
       }
       const int r0 = 4 * k;
       const int off = a * LS + ((r0 / CB) * 32 + lane) * CB + (r0 % CB);
       *reinterpret_cast<uint32_t*>(tab + off) = lo;
-      *reinterpret_cast<uint32_t*>(tab + A1 * LS + off) = hi;
+      if constexpr (SEQS == 2) *reinterpret_cast<uint32_t*>(tab + A1 * LS + off) = hi;
     }
   }
   __syncwarp();
@@ -859,6 +876,9 @@ __device__ __forceinline__ void emit_t(const TParams& p, uint32_t bb, int item) 
     if (hi >= limit) p.ovf_list[atomicAdd(p.ovf_count, 1)] = s1; else p.scores[p.perm[s1]] = hi;
   }
 }
+
+// exact 32-bit score of sequence position sq (T-mode recompute of a flagged sequence)
+__device__ __forceinline__ void emit_t32(const TParams& p, int score, int sq) { p.scores[p.perm[sq]] = score; }
 
 // One T-mode team (W warps) processing long pairs until the queue is exhausted.  first_item:
 // an item already taken for this team (or -1).  min_strips: a team of W warps only keeps items
@@ -930,21 +950,41 @@ struct TStream {
   int item[kTQ], base[kTQ], S[kTQ], rem[kTQ], mlo[kTQ], mhi[kTQ];
 };
 
-template <int C, class CC>
+// L = LaneS32: the 32-bit recompute of the flagged sequences (items = positions of
+// p.item_list, one sequence each; long-query mode, where the k_search recompute's query profile
+// does not fit shared memory).  Progress tags are 64-bit (running strip index << 32 | columns).
+template <int C, class L, class CC>
 __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uint8_t* tab,
                                               const int8_t* wp, int W, int team, int wt, int first_item,
-                                              uint32_t* prog, uint2* rb, TStream* ts) {
-  using L = LaneS16x2;
+                                              unsigned long long* prog, uint2* rb, TStream* ts) {
+  constexpr bool S32 = L::kSeqs == 1;
   constexpr int CB = chunk_bytes<C>();
   constexpr int LS = 32 * C;
   const int lane = threadIdx.x & 31;
   const int A1 = p.A_used + 1;
   const int qsteps = (p.qcols + 32 + 3) & ~3;
+  const int n_items = S32 ? *p.item_count : p.n_items;
   volatile TStream* vs = ts;
+  // item -> (pair, half): s16x2 items are pairs, s32 items index the flagged-sequence list
+  auto pair_of = [&](int item, int* half) {
+    if constexpr (S32) {
+      const int sq = p.item_list[item];
+      *half = sq & 1;
+      return sq >> 1;
+    } else {
+      *half = 0;
+      return item;
+    }
+  };
+  auto emit_item = [&](int item, int lo, int hi) {
+    if constexpr (S32) emit_t32(p, lo, p.item_list[item]);
+    else emit_t(p, ((uint32_t)lo & 0xffffu) | ((uint32_t)hi << 16), item);
+  };
   // append one pair to the ring (lane 0 of the warp holding the lock); empty pairs score 0
   auto append = [&](int item) {
-    const int S = (p.pair_ncols[item] + LS - 1) / LS;
-    if (S == 0) { emit_t(p, 0u, item); return; }
+    int hf;
+    const int S = (p.pair_ncols[pair_of(item, &hf)] + LS - 1) / LS;
+    if (S == 0) { emit_item(item, 0, 0); return; }
     const int k = vs->count % kTQ;
     if (vs->count >= kTQ)   // the entry kTQ pairs back must be finished before it is reused
       while (vs->rem[k] != 0) __nanosleep(64);
@@ -978,7 +1018,7 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
         if (atomicCAS(&ts->lock, 0, 1) == 0) {
           while (vs->next <= g && !vs->end) {
             const int item = p.gang_items + atomicAdd(p.work, 1);
-            if (item >= p.n_items) { vs->end = 1; break; }
+            if (item >= n_items) { vs->end = 1; break; }
             append(item);
           }
           __threadfence_block();
@@ -991,22 +1031,28 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
     k = __shfl_sync(SWB_FULL, k, 0);
     if (k < 0) break;
     const int item = vs->item[k], P = g - vs->base[k], S = vs->S[k];
-    const int ncols = p.pair_ncols[item];
-    const uint16_t* cp = p.cols + p.pair_off[item];
-    build_strip_tables<C>(p, tab, wp, cp, ncols, P);
+    int half;
+    const int pair = pair_of(item, &half);
+    const int ncols = p.pair_ncols[pair];
+    const uint16_t* cp = p.cols + p.pair_off[pair];
+    build_strip_tables<C, L::kSeqs>(p, tab, wp, cp, ncols, P, half);
     const int si = (g + W) % (W + 1), so = g % (W + 1);
-    uint32_t b = run_pass<L, 32, C, true, 4, false, 13>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps,
+    uint32_t b = run_pass<L, 32, C, true, 4, false, 32>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps,
                                                        P, S, rb + (int64_t)si * p.rb_cols + 1,
                                                        rb + (int64_t)so * p.rb_cols + 1, prog + si, prog + so, 0u, g);
 #pragma unroll
     for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
     if (lane == 0) {
-      atomicMax(&ts->mlo[k], (int)(int16_t)(b & 0xffffu));
-      atomicMax(&ts->mhi[k], (int)(int16_t)(b >> 16));
+      if constexpr (S32) {
+        atomicMax(&ts->mlo[k], (int)b);
+      } else {
+        atomicMax(&ts->mlo[k], (int)(int16_t)(b & 0xffffu));
+        atomicMax(&ts->mhi[k], (int)(int16_t)(b >> 16));
+      }
       __threadfence_block();
       if (atomicSub(&ts->rem[k], 1) == 1) {   // this pair's last strip
         const int lo = atomicAdd(&ts->mlo[k], 0), hi = atomicAdd(&ts->mhi[k], 0);
-        emit_t(p, ((uint32_t)lo & 0xffffu) | ((uint32_t)hi << 16), item);
+        emit_item(item, lo, hi);
       }
     }
     __syncwarp();
@@ -1064,19 +1110,20 @@ __device__ __forceinline__ void t_gang_item(const TParams& p, const CC& c, uint8
   }
 }
 
-template <int C, int NT, bool WIDE = false>
+template <int C, int NT, bool WIDE = false, class L = LaneS16x2>
 __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   constexpr int kWarps = NT / 32;
   constexpr int LS = 32 * C;
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ uint32_t sprog[2 * kWarps];
+  __shared__ unsigned long long sprog64[2 * kWarps];
   __shared__ uint32_t sred[kWarps];
   __shared__ int32_t sitem[kWarps];
   __shared__ int32_t sparked;
   // rows = the query's letters in compact order (row k = the k-th set bit of qmask) + the pad
   // row; columns = database letters (the database pad letter A maps to the pad value)
   const int A1 = p.A_used + 1;
-  const int table_bytes = 2 * A1 * LS;        // lo + hi tables of one warp
+  const int table_bytes = L::kSeqs * A1 * LS;  // lo (+ hi) tables of one warp
   // (A_used+1) rows of kWpStride bytes: w + rho for database letters d < A, -128 for the
   // database pad letter d == A (which is 32 for a 32-letter alphabet: the stride must exceed A)
   int8_t* wp = reinterpret_cast<int8_t*>(smem);
@@ -1107,7 +1154,9 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   // s % gang_ctas).  The CTA's first gang_warps warps (one per scheduler) work on that pair
   // while its other warps wait, so that the gang's dependency chain has its schedulers to
   // itself; then all warps go on to phase 2.
-  if (p.gang_items > 0) {
+  if constexpr (L::kSeqs == 1) {
+    // 32-bit recompute (long-query mode): the team stream only (no gangs, no whole-CTA phase)
+  } else if (p.gang_items > 0) {
     __shared__ int32_t sgslot;
     if (threadIdx.x == 0) sgslot = atomicAdd(p.gang_ctr, 1);
     __syncthreads();
@@ -1126,22 +1175,22 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   if (team >= nteams) return;
   const int first = (team == 0) ? sparked : -1;
   __shared__ TStream sts[kTmodeThreads / 32];
-  t_team_stream<C>(p, c, tab, wp, W, team, wt, first, sprog + team * (W + 1),
-                   rb_cta + (int64_t)team * (W + 1) * p.rb_cols, &sts[team]);
+  t_team_stream<C, L>(p, c, tab, wp, W, team, wt, first, sprog64 + team * (W + 1),
+                      rb_cta + (int64_t)team * (W + 1) * p.rb_cols, &sts[team]);
 }
 
-template <int C, int NT, bool WIDE>
+template <int C, int NT, bool WIDE, class L>
 cudaError_t launch_search_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st) {
-  k_search_t<C, NT, WIDE><<<grid, NT, smem_bytes, st>>>(p);
+  k_search_t<C, NT, WIDE, L><<<grid, NT, smem_bytes, st>>>(p);
   return cudaGetLastError();
 }
 
-template <int C, int NT, bool WIDE>
+template <int C, int NT, bool WIDE, class L>
 cudaError_t configure_tmode(int smem_bytes, int* blocks_per_sm) {
   cudaError_t e =
-      cudaFuncSetAttribute(k_search_t<C, NT, WIDE>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+      cudaFuncSetAttribute(k_search_t<C, NT, WIDE, L>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search_t<C, NT, WIDE>, NT, smem_bytes);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search_t<C, NT, WIDE, L>, NT, smem_bytes);
 }
 
 template <class L, int G, int Rs, int Rl, int NT, bool WIDE>

@@ -123,6 +123,8 @@ struct TParams {
   int32_t* scores;
   int32_t* ovf_list;
   int32_t* ovf_count;
+  const int32_t* item_list;  // 32-bit recompute (LaneS32 instantiation): flagged sequence positions
+  const int32_t* item_count; //   and their device count; the items of the team stream
   int32_t* work;
   int warps;                 // warps used per CTA (<= NT / 32, bounded by shared memory)
   int team_warps;            // warps per team in phase 2 (divides warps)
@@ -141,8 +143,8 @@ struct TParams {
   int32_t* gdone;            // gang_items: warps finished
 };
 
-cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st);
-cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm, bool wide);
+cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st, bool s32 = false);
+cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm, bool wide, bool s32 = false);
 cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, uint32_t qmask, cudaStream_t st);
 
 // Traceback of one pair (sw_traceback.cu): dir = m*n bytes, scratch = 7*m ints, result = 6 ints.

@@ -21,14 +21,23 @@ cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, uint32_t
   return cudaGetLastError();
 }
 
-cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st) {
-  if (p.delta > 0) return launch_search_tmode<kTmodeC, kTmodeThreads, true>(p, grid, smem_bytes, st);
-  return launch_search_tmode<kTmodeC, kTmodeThreads, false>(p, grid, smem_bytes, st);
+// s32 = true: the 32-bit recompute of the flagged sequences (p.item_list / p.item_count)
+cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st, bool s32) {
+  if (s32) {
+    if (p.delta > 0) return launch_search_tmode<kTmodeC, kTmodeThreads, true, LaneS32>(p, grid, smem_bytes, st);
+    return launch_search_tmode<kTmodeC, kTmodeThreads, false, LaneS32>(p, grid, smem_bytes, st);
+  }
+  if (p.delta > 0) return launch_search_tmode<kTmodeC, kTmodeThreads, true, LaneS16x2>(p, grid, smem_bytes, st);
+  return launch_search_tmode<kTmodeC, kTmodeThreads, false, LaneS16x2>(p, grid, smem_bytes, st);
 }
 
-cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm, bool wide) {
-  if (wide) return configure_tmode<kTmodeC, kTmodeThreads, true>(smem_bytes, blocks_per_sm);
-  return configure_tmode<kTmodeC, kTmodeThreads, false>(smem_bytes, blocks_per_sm);
+cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm, bool wide, bool s32) {
+  if (s32) {
+    if (wide) return configure_tmode<kTmodeC, kTmodeThreads, true, LaneS32>(smem_bytes, blocks_per_sm);
+    return configure_tmode<kTmodeC, kTmodeThreads, false, LaneS32>(smem_bytes, blocks_per_sm);
+  }
+  if (wide) return configure_tmode<kTmodeC, kTmodeThreads, true, LaneS16x2>(smem_bytes, blocks_per_sm);
+  return configure_tmode<kTmodeC, kTmodeThreads, false, LaneS16x2>(smem_bytes, blocks_per_sm);
 }
 
 }  // namespace swb

@@ -377,9 +377,8 @@ def test_maximum_query_and_sequence_lengths():
     """The limits include/sw.h declares: a query of SW_MAX_QUERY_LEN = 65536 residues over a
     2-letter alphabet (its profile fits SW_MAX_PROFILE_BYTES; many strips; one sequence holds
     an 8000-residue copy of it, so the s16 pass saturates and the 32-bit recompute decides),
-    the largest protein query the header guarantees (8192), a protein query of 65536 refused
-    with SW_E_UNSUPPORTED, and a database sequence of SW_MAX_SEQ_LEN = 1,048,512 residues in
-    both regimes."""
+    protein queries of 8192 (profile in shared memory) and 65536 (long-query mode), and a
+    database sequence of SW_MAX_SEQ_LEN = 1,048,512 residues in both regimes."""
     W2 = np.array([[5, -4], [-4, 5]], np.int8)
     q = (gen.u01(1007, "query", np.arange(1 << 16, dtype=np.uint64)) < 0.5).astype(np.uint8)
     parts = [(gen.u01(1043 + k, "res", np.arange(n, dtype=np.uint64)) < 0.5).astype(np.uint8)
@@ -399,9 +398,13 @@ def test_maximum_query_and_sequence_lengths():
     for T in (0, 3072):
         out, _ = _gpu(q, BLOSUM62, 10, 2, db, T)
         _assert_equal(out, ref, db, f"protein query 8192 T={T}")
-    with pytest.raises(swp.SWError) as e:
-        _gpu(gen.make_query(1 << 16, seed=7), BLOSUM62, 10, 2, db, 3072)
-    assert e.value.status == swp.SW_E_UNSUPPORTED
+    # a protein query of SW_MAX_QUERY_LEN residues: its profile exceeds shared memory, so the
+    # search runs in long-query mode (T-mode for every pair, tests/test_long_query_gpu.py)
+    q = gen.make_query(1 << 16, seed=7)
+    ref = _oracle(q, BLOSUM62, 10, 2, db)
+    out, st = _gpu(q, BLOSUM62, 10, 2, db, 3072)
+    _assert_equal(out, ref, db, "protein query 65536")
+    assert st["long_seqs"] == db.num_seqs
 
     q = gen.make_query(144)
     lmax = (1 << 20) - 64
