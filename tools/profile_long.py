@@ -1,0 +1,38 @@
+"""Drive searches of the LONG subset (n >= T) of a config's database with one query, the
+isolated long-regime launch of the threshold sweeps (for ncu captures of k_search_t).
+usage: python tools/profile_long.py [query_len=567] [T=3072] [reps=3] [config=C2] [env=K=V;...]"""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import numpy as np  # noqa: E402
+
+import paper_conf_ipps_hainscobr11_b200 as swp  # noqa: E402
+from workloads import gen  # noqa: E402
+from workloads.matrices import BLOSUM62  # noqa: E402
+
+m = int(sys.argv[1]) if len(sys.argv) > 1 else 567
+T = int(sys.argv[2]) if len(sys.argv) > 2 else 3072
+reps = int(sys.argv[3]) if len(sys.argv) > 3 else 3
+cfg = sys.argv[4] if len(sys.argv) > 4 else "C2"
+if len(sys.argv) > 5 and sys.argv[5]:
+    os.environ.update(dict(kv.split("=") for kv in sys.argv[5].split(";") if kv))
+if cfg == "C3":
+    lens = gen.long_lengths(4096, seed=3)
+    db = gen.build_database(lens, 3, None)
+else:
+    lens = gen.sp_lengths(540_000, seed=2)
+    db = gen.build_database(lens, 2, None)
+L = db.lengths
+idx = np.nonzero(L >= T)[0]
+off = np.concatenate([[0], np.cumsum(L[idx])]).astype(np.int64)
+res = np.concatenate([db.residues[db.offsets[i]:db.offsets[i + 1]] for i in idx])
+q = gen.make_query(m)
+with swp.SmithWaterman(q, BLOSUM62, 10, 2) as sw:
+    sw.load_db(res, off)
+    for _ in range(reps):
+        sw.search(T)
+        ms = sw.kernel_ms()["search_ms"]
+        print(f"{cfg} long subset n>={T}: {idx.size} seqs, {int(off[-1])} residues, m={m}: {ms:.3f} ms "
+              f"{m * int(off[-1]) / ms / 1e6:.0f} GCUPS", flush=True)
