@@ -51,10 +51,12 @@ enum {
 #define SW_MAX_ALPHABET 32          /* alphabet_size in [1, 32] */
 #define SW_MAX_QUERY_LEN (1 << 16)  /* 1 <= query_len <= 65536 (SW_E_INVALID beyond) */
 /* The int8 query profile (alphabet_size + 1 rows of query_len bytes, padded to the kernel's
- * strip layout) is staged whole in one CTA's shared memory; a search whose profile exceeds
- * SW_MAX_PROFILE_BYTES fails with SW_E_UNSUPPORTED (never a CPU fallback).  In practice:
- * query_len <= 8192 for the 24-letter protein alphabet (the paper's queries reach 5478),
- * query_len = 65536 for alphabets of up to 2 letters. */
+ * strip layout) is staged whole in one CTA's shared memory when it fits SW_MAX_PROFILE_BYTES
+ * (query_len up to ~8,900 for the 24-letter protein alphabet; the paper's queries reach 5478).
+ * Longer queries run in long-query mode: every database sequence takes the transposed
+ * long-sequence kernel, which streams the query from device memory and builds substitution
+ * tables per database strip (no query profile); the flagged sequences are recomputed by its
+ * 32-bit instantiation.  Same exact scores, every query length up to SW_MAX_QUERY_LEN. */
 #define SW_MAX_PROFILE_BYTES (220 * 1024)
 #define SW_MAX_SEQ_LEN ((1 << 20) - 64)  /* every database sequence length <= 1,048,512 */
 
@@ -65,9 +67,12 @@ enum {
 /* Create a handle for one query and one scoring scheme (§II: q, w, rho, sigma).
  *   query[query_len]      codes < alphabet_size, 1 <= query_len <= SW_MAX_QUERY_LEN
  *   matrix[A*A]           int8, row = query symbol, column = database symbol
- *   gap_open  (rho)       >= 0;  gap_extend (sigma) >= 0
- * Supported range: gap_open + max(matrix) <= 127 and gap_open + gap_extend <= 32000
- * (SW_E_UNSUPPORTED otherwise).
+ *   gap_open  (rho)       >= 0;  gap_extend (sigma) >= 0  (any int32 values; Eq.(1) bounds
+ *                         neither: rho + max(matrix) > 127 selects the WIDE kernels, whose
+ *                         int8 profile holds w + c with c < rho and adds rho - c per cell;
+ *                         penalties above 16384 are clamped for the 16-bit lanes with the
+ *                         overflow flag lowered to 16384, which is exact: DESIGN.md "Integer
+ *                         widths")
  * Uploads the query and builds the query profile on the device (§II-A). */
 int sw_create(sw_handle* out, const uint8_t* query, int32_t query_len,
               const int8_t* matrix, int32_t alphabet_size, int32_t gap_open, int32_t gap_extend);
@@ -111,11 +116,14 @@ int sw_search_batch_async(sw_handle h, const uint8_t* queries, const int64_t* q_
 /* Autotune (all search calls on a database loaded with sw_load_db): the first search of a
  * (query length, threshold) whose cells (query length x database residues) reach 1e10 times
  * the planner's 5 best kernel configurations, one search each, on the handle's first internal
- * stream, and keeps the fastest for later searches of that (query length, threshold).  That
- * first call therefore synchronises with the device (the async variants block for it) and
- * costs about five searches; its scores are the exact ones (every configuration computes the
- * same scores).  The table is cleared by sw_load_db.  Environment SW_AUTOTUNE=0 disables it
- * (the planner's model choice only). */
+ * stream, and keeps the fastest for later searches of that (query length, threshold).  With
+ * length_threshold == SW_AUTO_THRESHOLD the first search of a query length with >= 1e9 cells
+ * also times the threshold model's two best candidates and the all-short endpoint (plus the
+ * all-long one on databases whose sequences are all >= 512) and keeps the fastest threshold
+ * for that query length.  That first call therefore synchronises with the device (the async
+ * variants block for it) and costs a few searches; its scores are the exact ones (every
+ * configuration and threshold computes the same scores).  The tables are cleared by
+ * sw_load_db.  Environment SW_AUTOTUNE=0 disables both (the planner's model choices only). */
 
 /* Host-pointer variant of sw_search_batch_async (blocking; host int32[num_queries*num_seqs]). */
 int sw_search_batch(sw_handle h, const uint8_t* queries, const int64_t* q_offsets,

@@ -131,6 +131,10 @@ struct sw_handle_s {
   // measured plan choice per (query length, threshold) on the loaded database (run_batch
   // autotune; -1 = keep the model's choice); cleared by sw_load_db
   std::map<std::pair<int, int32_t>, int> tuned;
+  // measured automatic threshold per query length on the loaded database (run_batch autotune of
+  // SW_AUTO_THRESHOLD: the model's best candidates and the all-short endpoint, timed); cleared by
+  // sw_load_db
+  std::map<int, int64_t> tuned_T;
   int tune_force = -1;            // menu entry forced while tuning / from the tuned table
   std::vector<uint32_t> qmask;    // letters present in each query of the current batch
   // scratch
@@ -415,12 +419,24 @@ Split make_split(sw_handle h, int64_t T, int64_t* n_long_seqs_out) {
 // pairs run concurrently in T-mode at ~1.8x the group cost per cell (measured,
 // profiles/r01_sweep_*.jsonl).  Estimated time = max(throughput of both launches,
 // group tail / 0.8); the cheapest candidate wins (ties: the larger T).
+std::vector<std::pair<double, int64_t>> rank_thresholds(sw_handle h, int m);
+
 int64_t choose_threshold(sw_handle h, int m) {
+  if (h->db == &h->main_db) {
+    const auto it = h->tuned_T.find(m);
+    if (it != h->tuned_T.end()) return it->second;
+  }
+  const auto ranked = rank_thresholds(h, m);
+  return ranked.empty() ? 3072 : ranked.front().second;
+}
+
+// The candidates of choose_threshold with the model's estimated time, cheapest first (ties
+// within 0.5 %: the larger T, i.e. the candidate order).
+std::vector<std::pair<double, int64_t>> rank_thresholds(sw_handle h, int m) {
+  std::vector<std::pair<double, int64_t>> out;
   const int64_t maxlen = h->db->sorted_len.empty() ? 0 : h->db->sorted_len[0];
   const int64_t cands[] = {maxlen + 1, 16384, 12288, 8192, 6144, 4096, 3072, 2048, 1536, 1024, 768, 512};
   const std::string saved = h->err;
-  int64_t chosen = 3072;
-  double best = 1e300;
   // group cost per database column, from the plan with every pair in the group launch
   double per_col = 0.0;
   {
@@ -452,10 +468,14 @@ int64_t choose_threshold(sw_handle h, int m) {
     if (getenv("SW_DEBUG_AUTO"))
       fprintf(stderr, "auto m=%d T=%lld G=%d Rs=%d thr=%.3f long=%.3f tail=%.3f cost=%.3f ms\n", m, (long long)T,
               pl.cfg.G, pl.cfg.Rs, thr / 1.965e6, thr_long / 1.965e6, tail / 1.965e6, cost / 1.965e6);
-    if (cost < best * 0.995) { best = cost; chosen = T; }
+    out.emplace_back(cost, T);
   }
   h->err = saved;
-  return chosen;
+  // stable: equal (within 0.5 %) costs keep the candidate order, larger T first
+  std::stable_sort(out.begin(), out.end(), [](const std::pair<double, int64_t>& a, const std::pair<double, int64_t>& b) {
+    return a.first < b.first * 0.995;
+  });
+  return out;
 }
 
 // Long-query mode: the smallest query-profile image (the s32 recompute's team image, 32 lanes x
@@ -744,6 +764,8 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
           t.gang_items = items;
           t.gang_ctas = K;
           t.big_strips = 1 << 30;
+          t.gang_share = 1;
+          if (const char* f = getenv("SW_T_GANG_SHARE")) t.gang_share = atoi(f) != 0;
         }
       }
     }
@@ -976,6 +998,7 @@ int build_db(sw_handle h, DbState& db, const uint8_t* residues, const int64_t* o
 // candidates write the real output), and keeps the fastest for later searches.  SW_AUTOTUNE=0
 // disables it (model choice only); the tuned table is cleared by sw_load_db.
 constexpr double kTuneMinCells = 1e10;
+constexpr double kTuneTMinCells = 1e9;   // threshold tuning (3 searches of ~0.2 ms and up)
 constexpr int kTuneTop = 5;
 
 int autotune(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq, int32_t* d_out, int32_t T,
@@ -985,9 +1008,62 @@ int autotune(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq,
     if (!strcmp(f, "0")) return SW_OK;
   bool forked = false;
   const double residues = std::accumulate(h->db->sorted_len.begin(), h->db->sorted_len.end(), 0.0);
+  auto fork = [&]() -> int {
+    if (!forked) {   // the queries were uploaded on the caller's stream
+      SW_CUDA(h, cudaEventRecord(h->fork, user));
+      SW_CUDA(h, cudaStreamWaitEvent(h->slots[0].stream, h->fork, 0));
+      forked = true;
+    }
+    return SW_OK;
+  };
+  // one timed search of query k at threshold Tk with the plan enqueue_query makes (device ms
+  // of the search launches, profile build to join, on the first slot)
+  auto time_search = [&](int k, int32_t Tk, float* ms) -> int {
+    const int m = (int)(qoff[k + 1] - qoff[k]);
+    cudaEvent_t* ev = h->ev.data() + 3 * k;
+    int rc = enqueue_query(h, h->slots[0], d_queries + qoff[k], m, h->qmask[k], d_out + (int64_t)k * h->db->n_seqs,
+                           Tk, h->h_ovf + k, ev);
+    if (rc) return rc;
+    SW_CUDA(h, cudaEventSynchronize(ev[1]));
+    SW_CUDA(h, cudaEventElapsedTime(ms, ev[0], ev[1]));
+    return SW_OK;
+  };
   for (int k = 0; k < nq; ++k) {
     const int m = (int)(qoff[k + 1] - qoff[k]);
-    if ((double)m * residues < kTuneMinCells || long_query_mode(h, m)) continue;
+    if (long_query_mode(h, m)) continue;
+    // Automatic threshold: the model's estimate misses the occupancy of group
+    // launches with few items and the long path's tail, by up to 4x on long-sequence databases
+    // (C3 query 144).  The first search of a query length with
+    // SW_AUTO_THRESHOLD on a loaded database of >= kTuneTMinCells cells times the model's two
+    // best thresholds and the endpoints (all short: T > max length; all long: T = min length,
+    // for long-sequence databases) and keeps the fastest.
+    if (T == SW_AUTO_THRESHOLD && (double)m * residues >= kTuneTMinCells && !h->tuned_T.count(m)) {
+      const auto ranked = rank_thresholds(h, m);
+      std::vector<int64_t> cand;
+      for (const auto& c : ranked) {
+        if ((int)cand.size() >= 2) break;
+        cand.push_back(c.second);
+      }
+      const int64_t all_short = h->db->sorted_len.empty() ? 0 : h->db->sorted_len[0] + 1;
+      if (std::find(cand.begin(), cand.end(), all_short) == cand.end()) cand.push_back(all_short);
+      // the all-long endpoint only for databases of long sequences (C3-like: every sequence
+      // >= 512), where it is a real contender; on Swiss-Prot-like ones it is hopeless
+      const int64_t min_len = h->db->sorted_len.empty() ? 0 : h->db->sorted_len.back();
+      if (min_len >= 512 && std::find(cand.begin(), cand.end(), min_len) == cand.end()) cand.push_back(min_len);
+      int rc = fork();
+      if (rc) return rc;
+      float best_ms = 1e30f;
+      int64_t best_T = cand.front();
+      for (int64_t Tc : cand) {
+        float ms = 0.f;
+        rc = time_search(k, (int32_t)std::min<int64_t>(Tc, INT32_MAX), &ms);
+        if (rc) return rc;
+        if (getenv("SW_DEBUG_PLAN")) fprintf(stderr, "tune-T m=%d T=%lld %.3f ms\n", m, (long long)Tc, ms);
+        if (ms < best_ms) { best_ms = ms; best_T = Tc; }
+      }
+      h->tuned_T[m] = best_T;
+    }
+    if ((double)m * residues < kTuneMinCells) continue;
     int32_t Tk = T;
     if (Tk == SW_AUTO_THRESHOLD) Tk = (int32_t)std::min<int64_t>(choose_threshold(h, m), INT32_MAX);
     const std::pair<int, int32_t> key{m, Tk};
@@ -1003,23 +1079,16 @@ int autotune(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq,
     if (rc) return rc;
     std::sort(ranked.begin(), ranked.end());
     if (ranked.size() > (size_t)kTuneTop) ranked.resize(kTuneTop);
-    if (!forked) {   // the queries were uploaded on the caller's stream
-      SW_CUDA(h, cudaEventRecord(h->fork, user));
-      SW_CUDA(h, cudaStreamWaitEvent(h->slots[0].stream, h->fork, 0));
-      forked = true;
-    }
+    rc = fork();
+    if (rc) return rc;
     float best_ms = 1e30f;
     int best_i = -1;
     for (const auto& c : ranked) {
       h->tune_force = c.second;
-      cudaEvent_t* ev = h->ev.data() + 3 * k;
-      rc = enqueue_query(h, h->slots[0], d_queries + qoff[k], m, h->qmask[k], d_out + (int64_t)k * h->db->n_seqs, Tk,
-                         h->h_ovf + k, ev);
+      float ms = 0.f;
+      rc = time_search(k, Tk, &ms);
       h->tune_force = -1;
       if (rc) return rc;
-      SW_CUDA(h, cudaEventSynchronize(ev[1]));
-      float ms = 0.f;
-      SW_CUDA(h, cudaEventElapsedTime(&ms, ev[0], ev[1]));
       if (getenv("SW_DEBUG_PLAN")) fprintf(stderr, "tune m=%d T=%d menu=%d %.3f ms\n", m, (int)Tk, c.second, ms);
       if (ms < best_ms) { best_ms = ms; best_i = c.second; }
     }
@@ -1160,6 +1229,7 @@ int sw_load_db(sw_handle h, const uint8_t* residues, int64_t total_residues, con
   h->db = &h->main_db;
   h->main_db.release();
   h->tuned.clear();
+  h->tuned_T.clear();
   return build_db(h, h->main_db, residues, offsets, num_seqs, nullptr);
 }
 

@@ -1154,6 +1154,9 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   // s % gang_ctas).  The CTA's first gang_warps warps (one per scheduler) work on that pair
   // while its other warps wait, so that the gang's dependency chain has its schedulers to
   // itself; then all warps go on to phase 2.
+  // warps [wbase, p.warps) run the team stream; in a gang CTA with gang_share the gang's
+  // warps leave when their strips are done and the CTA's other warps stream meanwhile
+  int wbase = 0, W = p.team_warps;
   if constexpr (L::kSeqs == 1) {
     // 32-bit recompute (long-query mode): the team stream only (no gangs, no whole-CTA phase)
   } else if (p.gang_items > 0) {
@@ -1162,16 +1165,25 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
     __syncthreads();
     const int gi = sgslot / p.gang_ctas, rank = sgslot % p.gang_ctas;
     if (gi < p.gang_items) {
-      if (warp < p.gang_warps) t_gang_item<C>(p, c, tab, wp, gi, rank, warp);
-      __syncthreads();
+      if (p.gang_share) {
+        if (warp < p.gang_warps) {
+          t_gang_item<C>(p, c, tab, wp, gi, rank, warp);
+          return;
+        }
+        wbase = p.gang_warps;
+        W = min(W, p.warps - wbase);
+        while ((p.warps - wbase) % W) --W;
+      } else {
+        if (warp < p.gang_warps) t_gang_item<C>(p, c, tab, wp, gi, rank, warp);
+        __syncthreads();
+      }
     }
   } else if (p.warps > p.team_warps) {
     t_team_loop<C>(p, c, tab, wp, p.warps, 0, warp, -1, p.big_strips, &sparked, sprog, rb_cta, sitem, sred);
     __syncthreads();
   }
-  const int W = p.team_warps;
-  const int nteams = p.warps / W;
-  const int team = warp / W, wt = warp % W;
+  const int nteams = (p.warps - wbase) / W;
+  const int team = (warp - wbase) / W, wt = (warp - wbase) % W;
   if (team >= nteams) return;
   const int first = (team == 0) ? sparked : -1;
   __shared__ TStream sts[kTmodeThreads / 32];

@@ -136,6 +136,7 @@ struct TParams {
   // gangs (k_search_t phase 0): pairs [0, gang_items) are spread over gang_ctas CTAs x
   // gang_warps warps each; all buffers below are per gang pair and zeroed before the launch
   int gang_items, gang_ctas, gang_warps;
+  int gang_share;            // 1: the gang CTAs' other warps run the team stream meanwhile
   int32_t* gang_ctr;         // slot counter
   uint32_t* gprog;           // gang_items x (GW + 1) progress flags, GW = gang_ctas * gang_warps
   uint2* grb;                // gang_items x (GW + 1) x rb_cols row buffers

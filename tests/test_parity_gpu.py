@@ -109,9 +109,10 @@ def test_long_sequence_modes(mode, m):
         _assert_equal(out, ref, db, f"mode={mode} m={m} T={T}")
 
 
+@pytest.mark.parametrize("share", ["0", "1"])
 @pytest.mark.parametrize("gang", ["2", "3", "8", "2:1", "5:3"])
 @pytest.mark.parametrize("m", [1, 144, 1500])
-def test_tmode_gangs(gang, m):
+def test_tmode_gangs(gang, m, share):
     """T-mode gangs: the longest pairs spread over K CTAs (strip pipeline across CTAs through
     global row buffers and gpu-scope progress flags), SW_T_GANG = "K" (every long pair) or
     "K:items" (the items longest pairs); the other pairs take the CTA teams."""
@@ -122,7 +123,8 @@ def test_tmode_gangs(gang, m):
     q = gen.make_query(m, seed=990 + m)
     ref = _oracle(q, BLOSUM62, 10, 2, db)
     for T in (0, 3000):
-        out, _ = _gpu(q, BLOSUM62, 10, 2, db, T, env={"SW_LONG_MODE": "t", "SW_T_GANG": gang})
+        out, _ = _gpu(q, BLOSUM62, 10, 2, db, T, env={"SW_LONG_MODE": "t", "SW_T_GANG": gang,
+                                                      "SW_T_GANG_SHARE": share})
         _assert_equal(out, ref, db, f"gang={gang} m={m} T={T}")
 
 
