@@ -764,7 +764,10 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
           t.gang_items = items;
           t.gang_ctas = K;
           t.big_strips = 1 << 30;
-          t.gang_share = 1;
+          // the gang CTAs' other warps wait (measured: letting them stream meanwhile slows the
+          // gang's latency-bound strip pipeline more than it gains: C2 query 567 long-only at
+          // T = 3072 1.156 -> 1.359 ms, profiles/r02_gang_share.txt); SW_T_GANG_SHARE=1 for A/B
+          t.gang_share = 0;
           if (const char* f = getenv("SW_T_GANG_SHARE")) t.gang_share = atoi(f) != 0;
         }
       }
@@ -784,6 +787,8 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
       t.gprog = reinterpret_cast<uint32_t*>(s.d_gang + 1 + 3 * t.gang_items);
       t.grb = s.d_grb;
     }
+    t.two_col = 1;
+    if (const char* f = getenv("SW_T_TWO_COL")) t.two_col = atoi(f) != 0;
     t.rb = s.d_rb_t;
     t.rb_cols = qcols + kPadCols + 1;
     t.hi_mul = 1u << 24;
