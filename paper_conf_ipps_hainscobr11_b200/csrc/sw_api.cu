@@ -787,8 +787,6 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
       t.gprog = reinterpret_cast<uint32_t*>(s.d_gang + 1 + 3 * t.gang_items);
       t.grb = s.d_grb;
     }
-    t.two_col = 1;
-    if (const char* f = getenv("SW_T_TWO_COL")) t.two_col = atoi(f) != 0;
     t.rb = s.d_rb_t;
     t.rb_cols = qcols + kPadCols + 1;
     t.hi_mul = 1u << 24;

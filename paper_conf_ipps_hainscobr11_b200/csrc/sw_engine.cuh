@@ -435,180 +435,6 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
   return best;
 }
 
-// Two columns per step (run_pass2): the cell update of columns A = j and B = j + 1 for the
-// lane's R rows, interleaved with a one-row skew — row r of A, then row r - 1 of B — so that two
-// independent vertical chains (f -> h -> hr -> f, ~13 cycles per row through the FMA pipe) are
-// in flight in one warp: the ncu stall profile of the one-column step is dominated by that
-// chain's fixed-latency waits (T-mode: "wait" 1.25 per issue, 2 warps per scheduler).  Row r of
-// B needs e[r] and t[r] as column A left them (E[r][B] and H[r-1][A] + w(q_r, d_B)) and the
-// vertical values of its own row r - 1, all available one row-step earlier.  wA: profile words
-// of column B's letters (the diagonal term A forms for B), wB: those of column B + 1 (for the
-// next step's column A).  Same instructions per cell as cell_rows; per-column overheads of the
-// step (loop, rings, publication) are shared by two columns.
-template <class L, int R, bool WIDE = false>
-__device__ __forceinline__ void cell_rows2(uint32_t (&e)[R], uint32_t (&t)[R],
-                                           const uint32_t (&wloA)[(R + 3) / 4], const uint32_t (&whiA)[(R + 3) / 4],
-                                           const uint32_t (&wloB)[(R + 3) / 4], const uint32_t (&whiB)[(R + 3) / 4],
-                                           uint32_t nrho, uint32_t prho, uint32_t nsig, uint32_t& hupA, uint32_t& fsA,
-                                           uint32_t& hupB, uint32_t& fsB, uint32_t& best, uint32_t dlt = 0u) {
-  uint32_t hrupA = L::add(hupA, nrho), fA = L::add(fsA, nrho), hA = 0;
-  uint32_t hrupB = L::add(hupB, nrho), fB = L::add(fsB, nrho), hB = 0;
-#pragma unroll
-  for (int r = 0; r <= R; ++r) {
-    const uint32_t hAprev = hA;   // row r - 1 of A, folded into best with row r - 1 of B
-    if (r < R) {   // column A, row r
-      fA = L::gap(fA, nsig, hrupA);
-      hA = L::hmax(t[r], e[r], fA);
-      const uint32_t hr = L::add(hA, nrho);
-      e[r] = L::gap(e[r], nsig, hr);
-      t[r] = L::add(WIDE ? L::add(hrupA, dlt) : hrupA, subst_row<L, R>(wloA, whiA, r));
-      hrupA = hr;
-    }
-    if (r >= 1) {  // column B, row r - 1
-      const int q = r - 1;
-      fB = L::gap(fB, nsig, hrupB);
-      hB = L::hmax(t[q], e[q], fB);
-      const uint32_t hr = L::add(hB, nrho);
-      e[q] = L::gap(e[q], nsig, hr);
-      t[q] = L::add(WIDE ? L::add(hrupB, dlt) : hrupB, subst_row<L, R>(wloB, whiB, q));
-      hrupB = hr;
-      best = L::max3(best, hAprev, hB);
-    }
-  }
-  hupA = hA;
-  fsA = L::add(fA, prho);
-  hupB = hB;
-  fsB = L::add(fB, prho);
-}
-
-// run_pass with two columns per step (cell_rows2): lane l processes columns jA = 2(s - l) - 2
-// and jB = jA + 1 at step s; lane 0's inputs (residues one column ahead, the previous strip's
-// bottom row) come through 4-step register rings as in run_pass (8 columns per group).  steps
-// counts double steps: a multiple of 4 with 2 * (steps - GC) >= ncols.  Used by T-mode (team
-// stream, whole-CTA teams, gangs), where the chain latency rather than the ALU pipe bounds the
-// one-column step.
-template <class L, int GC, int R, bool TEAM, int PUB = 4, bool GPU_FLAGS = false, int TAG_SHIFT = 20,
-          class CC = ChainConst, class TagT = uint32_t>
-__device__ __forceinline__ uint32_t run_pass2(const CC& c, const uint8_t* prow, int ls, int hi_off,
-                                              const uint16_t* __restrict__ cols, int ncols, int steps, int P,
-                                              int passes_total, const uint2* __restrict__ rb_in,
-                                              uint2* __restrict__ rb_out, const TagT* prog_in, TagT* prog_out,
-                                              uint32_t best, int tagP = -1) {
-  static_assert(TAG_SHIFT < 8 * (int)sizeof(TagT), "tag type too narrow");
-  const TagT tag_base = (TagT)(tagP >= 0 ? tagP : P) << TAG_SHIFT;
-  const TagT tag_prev = tag_base - ((TagT)1 << TAG_SHIFT);
-  const int lane = threadIdx.x & 31;
-  const int gl = lane & (GC - 1);
-  const uint32_t nrho = L::splat(-c.rho), prho = L::splat(c.rho);
-  const uint32_t nsig = L::splat(-c.sigma);
-  const uint32_t dlt = L::splat(c.delta);
-  constexpr int CB = chunk_bytes<R>();
-  const bool store_out = (gl == GC - 1) && (P < passes_total - 1);
-  const bool from_prev = P > 0;
-
-  uint32_t e[R], t[R];
-#pragma unroll
-  for (int r = 0; r < R; ++r) { e[r] = nrho; t[r] = 0u; }
-  uint32_t yA_hr = 0, yA_f = 0, yB_hr = 0, yB_f = 0, yA_res = c.padpair, yB_res = c.padpair;
-  int col = -2 * gl - 2;   // column A of this lane at the current step
-  const int cmax = ncols + kPadCols - 1;
-  const int rlast = 2 * (steps - GC) - 1;   // the last column the previous strip's last lane wrote
-  // rings: per step k of a group, residues of columns c0 + 2k + 1 and + 2 (look-ahead) and the
-  // previous strip's bottom row at columns c0 + 2k and + 1
-  uint32_t raA[4], raB[4], rhA[4], rfA[4], rhB[4], rfB[4];
-  uint32_t sbA[4], sbB[4], shA[4], sfA[4], shB[4], sfB[4];
-#pragma unroll
-  for (int k = 0; k < 4; ++k) {
-    rhA[k] = rfA[k] = rhB[k] = rfB[k] = shA[k] = sfA[k] = shB[k] = sfB[k] = 0;
-    raA[k] = raB[k] = sbA[k] = sbB[k] = c.padpair;
-  }
-  TagT known = 0;
-  auto fetch_group = [&](uint32_t (&ra)[4], uint32_t (&rb)[4], uint32_t (&rh)[4], uint32_t (&rf)[4],
-                         uint32_t (&rh2)[4], uint32_t (&rf2)[4], int c0) {
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {   // (column -1 of the first group: the pad letter)
-      const int i = c0 + 2 * k + 1;
-      ra[k] = i >= 0 ? (uint32_t)cols[min(i, cmax)] : c.padpair;
-      rb[k] = cols[min(i + 1, cmax)];
-    }
-    if (from_prev) {
-      if constexpr (TEAM) {
-        const TagT need = tag_prev | (TagT)(min(c0 + 7, rlast) + 1);
-        while (known < need) {
-          if constexpr (GPU_FLAGS) known = ld_acquire_gpu(prog_in);
-          else known = ld_acquire_smem(prog_in);
-          if (known < need) __nanosleep(32);
-        }
-      }
-#pragma unroll
-      for (int k = 0; k < 4; ++k) {   // (index -1: the neutral leading entry)
-        const uint2 v = rb_in[max(min(c0 + 2 * k, rlast), -1)];
-        const uint2 u = rb_in[min(c0 + 2 * k + 1, rlast)];
-        rh[k] = v.x; rf[k] = v.y; rh2[k] = u.x; rf2[k] = u.y;
-      }
-    }
-  };
-  auto step = [&](auto kc, const uint32_t (&ra)[4], const uint32_t (&rb)[4], const uint32_t (&rh)[4],
-                  const uint32_t (&rf)[4], const uint32_t (&rh2)[4], const uint32_t (&rf2)[4]) {
-    constexpr int K = decltype(kc)::value;
-    uint32_t xA_hr = __shfl_up_sync(SWB_FULL, yA_hr, 1, GC);
-    uint32_t xA_f = __shfl_up_sync(SWB_FULL, yA_f, 1, GC);
-    uint32_t xB_hr = __shfl_up_sync(SWB_FULL, yB_hr, 1, GC);
-    uint32_t xB_f = __shfl_up_sync(SWB_FULL, yB_f, 1, GC);
-    uint32_t xA_res = __shfl_up_sync(SWB_FULL, yA_res, 1, GC);
-    uint32_t xB_res = __shfl_up_sync(SWB_FULL, yB_res, 1, GC);
-    if (gl == 0) {
-      xA_hr = rh[K]; xA_f = rf[K]; xB_hr = rh2[K]; xB_f = rf2[K]; xA_res = ra[K]; xB_res = rb[K];
-    }
-    uint32_t wloA[(R + 3) / 4], whiA[(R + 3) / 4], wloB[(R + 3) / 4], whiB[(R + 3) / 4];
-    {
-      const int ahA = (int)__umulhi(xA_res, c.hi_mul), ahB = (int)__umulhi(xB_res, c.hi_mul);
-      const int ohA = ahA * ls, ohB = ahB * ls;
-      load_prof<R, CB, GC * CB>(wloA, prow + ((int)xA_res * ls - ohA * 256));
-      load_prof<R, CB, GC * CB>(wloB, prow + ((int)xB_res * ls - ohB * 256));
-      if constexpr (L::kSeqs == 2) {
-        load_prof<R, CB, GC * CB>(whiA, prow + hi_off + ohA);
-        load_prof<R, CB, GC * CB>(whiB, prow + hi_off + ohB);
-      }
-    }
-    uint32_t hA = xA_hr, fA = xA_f, hB = xB_hr, fB = xB_f;
-    cell_rows2<L, R, CC::kWide>(e, t, wloA, whiA, wloB, whiB, nrho, prho, nsig, hA, fA, hB, fB, best, dlt);
-    yA_hr = hA; yA_f = fA; yB_hr = hB; yB_f = fB; yA_res = xA_res; yB_res = xB_res;
-    if (store_out) {
-      rb_out[max(col, -1)] = make_uint2(hA, fA);
-      rb_out[max(col + 1, -1)] = make_uint2(hB, fB);
-    }
-    col += 2;
-  };
-  auto publish = [&]() {
-    if (TEAM && store_out) {
-      const int done = col;   // the last lane's columns < col are stored
-      if (done > 0 && (PUB == 4 || (done & 15) < 8 || done > rlast)) {
-        if constexpr (GPU_FLAGS) st_release_gpu(prog_out, tag_base | (TagT)min(done, rlast + 1));
-        else st_release_smem(prog_out, tag_base | (TagT)min(done, rlast + 1));
-      }
-    }
-  };
-  // lane 0's column A at step s is 2s - 2
-  fetch_group(raA, raB, rhA, rfA, rhB, rfB, -2);
-  for (int s = 0; s < steps; s += 8) {
-    fetch_group(sbA, sbB, shA, sfA, shB, sfB, 2 * (s + 4) - 2);
-    step(std::integral_constant<int, 0>{}, raA, raB, rhA, rfA, rhB, rfB);
-    step(std::integral_constant<int, 1>{}, raA, raB, rhA, rfA, rhB, rfB);
-    step(std::integral_constant<int, 2>{}, raA, raB, rhA, rfA, rhB, rfB);
-    step(std::integral_constant<int, 3>{}, raA, raB, rhA, rfA, rhB, rfB);
-    publish();
-    if (s + 4 >= steps) break;
-    fetch_group(raA, raB, rhA, rfA, rhB, rfB, 2 * (s + 8) - 2);
-    step(std::integral_constant<int, 0>{}, sbA, sbB, shA, sfA, shB, sfB);
-    step(std::integral_constant<int, 1>{}, sbA, sbB, shA, sfA, shB, sfB);
-    step(std::integral_constant<int, 2>{}, sbA, sbB, shA, sfA, shB, sfB);
-    step(std::integral_constant<int, 3>{}, sbA, sbB, shA, sfA, shB, sfB);
-    publish();
-  }
-  return best;
-}
-
 // emit the score(s) of one chain result; s16x2: both sequences of the pair
 template <class L>
 __device__ __forceinline__ void emit(const SearchParams& p, uint32_t b, int pair, int half) {
@@ -1070,7 +896,6 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const CC& c, uint8
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int A1 = p.A_used + 1;                 // compact query letters + the pad row
   const int qsteps = (p.qcols + 32 + 3) & ~3;
-  const int qsteps2 = (p.qcols / 2 + 32 + 3) & ~3;   // run_pass2: double steps, 2 * (qsteps2 - 32) >= qcols
   int pending = first_item;
   for (;;) {
     team_bar(team, W);
@@ -1094,14 +919,9 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const CC& c, uint8
     for (int P = wt; P < S; P += W) {
       build_strip_tables<C>(p, tab, wp, cp, ncols, P);
       const int si = (P + W) % (W + 1), so = P % (W + 1);
-      if (p.two_col)
-      b = run_pass2<L, 32, C, true, 4>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, qsteps2, P, S,
-                                        rb + (int64_t)si * p.rb_cols + 1, rb + (int64_t)so * p.rb_cols + 1, prog + si,
-                                        prog + so, b);
-    else
       b = run_pass<L, 32, C, true, 4>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps, P, S,
-                                       rb + (int64_t)si * p.rb_cols + 1, rb + (int64_t)so * p.rb_cols + 1, prog + si,
-                                       prog + so, b);
+                                     rb + (int64_t)si * p.rb_cols + 1, rb + (int64_t)so * p.rb_cols + 1, prog + si,
+                                     prog + so, b);
     }
 #pragma unroll
     for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
@@ -1143,7 +963,6 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
   const int lane = threadIdx.x & 31;
   const int A1 = p.A_used + 1;
   const int qsteps = (p.qcols + 32 + 3) & ~3;
-  const int qsteps2 = (p.qcols / 2 + 32 + 3) & ~3;   // run_pass2: double steps, 2 * (qsteps2 - 32) >= qcols
   const int n_items = S32 ? *p.item_count : p.n_items;
   volatile TStream* vs = ts;
   // item -> (pair, half): s16x2 items are pairs, s32 items index the flagged-sequence list
@@ -1218,15 +1037,9 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
     const uint16_t* cp = p.cols + p.pair_off[pair];
     build_strip_tables<C, L::kSeqs>(p, tab, wp, cp, ncols, P, half);
     const int si = (g + W) % (W + 1), so = g % (W + 1);
-    uint32_t b;
-    if (p.two_col)
-      b = run_pass2<L, 32, C, true, 4, false, 32>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, qsteps2, P, S,
-                                                  rb + (int64_t)si * p.rb_cols + 1, rb + (int64_t)so * p.rb_cols + 1,
-                                                  prog + si, prog + so, 0u, g);
-    else
-      b = run_pass<L, 32, C, true, 4, false, 32>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps, P, S,
-                                                 rb + (int64_t)si * p.rb_cols + 1, rb + (int64_t)so * p.rb_cols + 1,
-                                                 prog + si, prog + so, 0u, g);
+    uint32_t b = run_pass<L, 32, C, true, 4, false, 32>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps,
+                                                       P, S, rb + (int64_t)si * p.rb_cols + 1,
+                                                       rb + (int64_t)so * p.rb_cols + 1, prog + si, prog + so, 0u, g);
 #pragma unroll
     for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
     if (lane == 0) {
@@ -1268,7 +1081,6 @@ __device__ __forceinline__ void t_gang_item(const TParams& p, const CC& c, uint8
   const int lane = threadIdx.x & 31;
   const int A1 = p.A_used + 1;
   const int qsteps = (p.qcols + 32 + 3) & ~3;
-  const int qsteps2 = (p.qcols / 2 + 32 + 3) & ~3;   // run_pass2: double steps, 2 * (qsteps2 - 32) >= qcols
   const int GW = p.gang_ctas * p.gang_warps;
   const int gw = rank * p.gang_warps + warp;
   const int ncols = p.pair_ncols[gi];
@@ -1280,14 +1092,9 @@ __device__ __forceinline__ void t_gang_item(const TParams& p, const CC& c, uint8
   for (int P = gw; P < S; P += GW) {
     build_strip_tables<C>(p, tab, wp, cp, ncols, P);
     const int si = (P + GW) % (GW + 1), so = P % (GW + 1);
-    if (p.two_col)
-      b = run_pass2<L, 32, C, true, 16, true>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, qsteps2, P, S,
-                                               rb + (int64_t)si * p.rb_cols + 1, rb + (int64_t)so * p.rb_cols + 1,
-                                               prog + si, prog + so, b);
-    else
-      b = run_pass<L, 32, C, true, 16, true>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps, P, S,
-                                            rb + (int64_t)si * p.rb_cols + 1, rb + (int64_t)so * p.rb_cols + 1,
-                                            prog + si, prog + so, b);
+    b = run_pass<L, 32, C, true, 16, true>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps, P, S,
+                                          rb + (int64_t)si * p.rb_cols + 1, rb + (int64_t)so * p.rb_cols + 1,
+                                          prog + si, prog + so, b);
   }
 #pragma unroll
   for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));

@@ -137,7 +137,6 @@ struct TParams {
   // gang_warps warps each; all buffers below are per gang pair and zeroed before the launch
   int gang_items, gang_ctas, gang_warps;
   int gang_share;            // 1: the gang CTAs' other warps run the team stream meanwhile
-  int two_col;               // 1: two query columns per step (run_pass2, cell_rows2)
   int32_t* gang_ctr;         // slot counter
   uint32_t* gprog;           // gang_items x (GW + 1) progress flags, GW = gang_ctas * gang_warps
   uint2* grb;                // gang_items x (GW + 1) x rb_cols row buffers

@@ -97,6 +97,33 @@ def sp_lengths(n_seqs: int, seed: int, mu: float = 5.5219, sigma: float = 0.8262
     return n
 
 
+VARIANCE_STDS = [100, 250, 500, 1000, 2000, 4000]
+
+
+def variance_lengths(n_seqs: int, std: float, seed: int, max_len: int = 60000) -> np.ndarray:
+    """Length-variance workload (Fig.2, L16 §II-C): log-normal lengths with standard
+    deviation `std` and mean 1000 + std ("the mean varies" with the deviation), clipped to
+    [2, max_len]."""
+    mean = 1000.0 + std
+    s2 = np.log1p((std / mean) ** 2)
+    mu = np.log(mean) - s2 / 2
+    z = normal(seed, "len", np.arange(n_seqs, dtype=np.uint64))
+    return np.clip(np.rint(np.exp(mu + np.sqrt(s2) * z)), 2, max_len).astype(np.int64)
+
+
+# PAPER.md L28-L30 Table II: fraction of sequences above T = 3072 (reading c19: ".53%" = 0.53 %)
+TABLE2 = [("Ensembl Dog", 0.0053), ("Ensembl Rat", 0.0035), ("RefSeq Human", 0.0056),
+          ("RefSeq Mouse", 0.0054), ("TAIR", 0.0006), ("Swiss-Prot", 0.0012)]
+
+
+def table2_lengths(n_seqs: int, frac_over_3072: float, seed: int) -> np.ndarray:
+    """Log-normal lengths with Swiss-Prot's median (mu = 5.5219) and the sigma that puts
+    `frac_over_3072` of the sequences at n >= 3072 (one Table II database shape)."""
+    from scipy.stats import norm
+    sigma = (np.log(3072.0) - 5.5219) / norm.ppf(1.0 - frac_over_3072)
+    return sp_lengths(n_seqs, seed, mu=5.5219, sigma=float(sigma), tail_frac=0.0)
+
+
 def long_lengths(n_seqs: int, seed: int, lo: int = 3073, max_len: int = MAX_LEN,
                  mu: float = 5.5219, sigma: float = 0.8262) -> np.ndarray:
     """Config 3: 90% SP log-normal truncated to [lo, max] by rejection, 10% log-uniform
