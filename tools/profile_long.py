@@ -1,6 +1,7 @@
 """Drive searches of the LONG subset (n >= T) of a config's database with one query, the
 isolated long-regime launch of the threshold sweeps (for ncu captures of k_search_t).
-usage: python tools/profile_long.py [query_len=567] [T=3072] [reps=3] [config=C2] [env=K=V;...]"""
+usage: python tools/profile_long.py [query_len=567] [T=3072] [reps=3] [config=C2] [env=K=V;...] [top:K|drop:K]
+(top:K keeps only the K longest sequences of the subset, drop:K removes them)"""
 import os
 import sys
 
@@ -26,6 +27,10 @@ else:
     db = gen.build_database(lens, 2, None)
 L = db.lengths
 idx = np.nonzero(L >= T)[0]
+if len(sys.argv) > 6 and sys.argv[6]:
+    mode, k = sys.argv[6].split(":")
+    order = idx[np.argsort(-L[idx], kind="stable")]
+    idx = np.sort(order[:int(k)] if mode == "top" else order[int(k):])
 off = np.concatenate([[0], np.cumsum(L[idx])]).astype(np.int64)
 res = np.concatenate([db.residues[db.offsets[i]:db.offsets[i + 1]] for i in idx])
 q = gen.make_query(m)
