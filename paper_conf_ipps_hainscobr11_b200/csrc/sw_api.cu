@@ -148,6 +148,7 @@ struct sw_handle_s {
   // on each other, so two gang launches must never hold SMs at the same time; sw_engine.cuh
   // t_gang_item)
   cudaEvent_t gang_ev = nullptr;
+  uint32_t gang_epoch = 0;        // tag epoch of the last gang launch (sw_engine.cuh run_pass GPU_FLAGS)
   // stats
   int64_t stat_long = 0, stat_short = 0, stat_launches = 0;
   int stat_nq = 0;
@@ -777,9 +778,19 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
       const size_t ints = 1 + 3 * (size_t)t.gang_items + (size_t)t.gang_items * (GW + 1);
       rc = grow(h, &s.d_gang, &s.gang_cap, ints * sizeof(int32_t), "alloc gang scratch", tst);
       if (rc) return rc;
-      rc = grow(h, &s.d_grb, &s.grb_cap, (size_t)t.gang_items * (GW + 1) * (qcols + kPadCols + 1) * sizeof(uint2),
-                "alloc gang row buffers", tst, true);
+      const size_t grb_bytes = (size_t)t.gang_items * (GW + 1) * (qcols + kPadCols + 1) * 2 * sizeof(uint2);
+      rc = grow(h, &s.d_grb, &s.grb_cap, grb_bytes, "alloc gang row buffers", tst, true);
       if (rc) return rc;
+      // hand-off words are tagged with a launch epoch: a word left by an earlier launch never
+      // matches (cleared when the 20-bit epoch wraps)
+      h->gang_epoch = (h->gang_epoch + 1) & 0xfffff;
+      if (h->gang_epoch == 0) {
+        SW_CUDA(h, cudaMemsetAsync(s.d_grb, 0, s.grb_cap, tst));
+        h->gang_epoch = 1;
+      }
+      t.gang_epoch = h->gang_epoch;
+      t.gang_chain2 = 1;
+      if (const char* f = getenv("SW_T_GANG_CHAIN2")) t.gang_chain2 = atoi(f) != 0;
       SW_CUDA(h, cudaMemsetAsync(s.d_gang, 0, ints * sizeof(int32_t), tst));
       t.gang_ctr = s.d_gang;
       t.gbest = s.d_gang + 1;

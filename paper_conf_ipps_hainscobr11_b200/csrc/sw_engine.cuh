@@ -159,6 +159,17 @@ __device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
 __device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
+// tagged hand-off words (T-mode gangs): one 64-bit word = (tag << 32) | value, written and read
+// as single-copy-atomic relaxed gpu-scope accesses, so a reader that sees the tag of the strip
+// it waits for sees that strip's value (no release fence, no separate flag)
+__device__ __forceinline__ unsigned long long ld_relaxed_gpu_u64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed_gpu_u64(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
 __device__ __forceinline__ void team_bar(int team, int W) {
   if (W > 1) {
     asm volatile("bar.sync %0, %1;" ::"r"(team + 1), "r"(W * 32) : "memory");
@@ -258,11 +269,36 @@ using ChainConst = ChainConstT<false>;
 // pair and measured 4-5 % slower: issue slots, not the chain, are the tighter limit.)
 // Vertical values enter and leave as (H, F + rho), the format of the lane hand-off and of the
 // strip row buffers.
-template <class L, int R, bool WIDE = false>
+// CHAIN2 ("u form", for latency-bound warps: the T-mode gangs, one warp per scheduler): the
+// vertical chain is two ALU ops per row instead of three (through the FMA pipe):
+//   g    = max(g - sigma, h_up)     F + rho, directly in the hand-off format   VIADDMNMX
+//   u    = max(t[r], e[r], 0)       off the chain                               VIMNMX3.RELU
+//   h    = max(g - rho, u)          H                                           VIADDMNMX
+// at one more ALU-pipe instruction per cell pair (5.5 instead of 4.5; the t form wins where
+// the ALU pipe, not the chain, is the limit — every throughput-bound launch).
+template <class L, int R, bool WIDE = false, bool CHAIN2 = false>
 __device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&t)[R], const uint32_t (&wlo)[(R + 3) / 4],
                                           const uint32_t (&whi)[(R + 3) / 4], uint32_t nrho, uint32_t prho,
                                           uint32_t nsig, uint32_t& hup, uint32_t& fs, uint32_t& best,
                                           uint32_t dlt = 0u) {
+  if constexpr (CHAIN2) {
+    uint32_t hrup = L::add(hup, nrho), g = fs, h = hup, hprev = 0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const uint32_t u = L::hmax(t[r], e[r], e[r]);                  // max(H[i-1][j-1] + w, E, 0)
+      g = L::gap(g, nsig, h);                                         // F + rho = max(F[i-1] + rho - sigma, H[i-1])
+      h = L::gap(g, nrho, u);                                         // H = max(F, u)
+      const uint32_t hr = L::add(h, nrho);
+      e[r] = L::gap(e[r], nsig, hr);
+      t[r] = L::add(WIDE ? L::add(hrup, dlt) : hrup, subst_row<L, R>(wlo, whi, r));
+      hrup = hr;
+      if (r & 1) best = L::max3(best, hprev, h); else hprev = h;
+    }
+    if constexpr (R & 1) best = L::max2(best, hprev);
+    hup = h;
+    fs = g;
+    return;
+  }
   uint32_t hrup = L::add(hup, nrho), f = L::add(fs, nrho), hprev = 0, h = 0;
 #pragma unroll
   for (int r = 0; r < R; ++r) {
@@ -292,14 +328,19 @@ __device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&t)[R], co
 // neutral fill values).  Returns max(best, this lane's H maxima) (packed per Lane).
 // ONE_PASS: the query is one strip (no row buffer in or out): the first lane's top input is
 // the constant boundary (0, 0), so the boundary rings and their loads disappear (registers).
+// GPU_FLAGS (T-mode gangs, strips on different SMs): the row buffers hold two tagged 64-bit
+// words per column, (tag << 32 | H) and (tag << 32 | F + rho) with tag = epoch << 12 | (P + 1),
+// written by the producing strip's last lane as it goes; the consuming strip's lane 0 polls
+// the words it needs (a per-column "flag in the data": no release fence, no progress flag,
+// no publication granularity).  prog_in / prog_out are unused then.
 template <class L, int GC, int R, bool TEAM, int PUB = 16, bool GPU_FLAGS = false, int TAG_SHIFT = 20,
-          bool ONE_PASS = false, class CC = ChainConst, class TagT = uint32_t>
+          bool ONE_PASS = false, bool CHAIN2 = false, class CC = ChainConst, class TagT = uint32_t>
 __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, int ls, int hi_off,
                                              const uint16_t* __restrict__ cols, int ncols,
                                              int half, int steps, int P, int passes_total,
                                              const uint2* __restrict__ rb_in, uint2* __restrict__ rb_out,
                                              const TagT* prog_in, TagT* prog_out, uint32_t best,
-                                             int tagP = -1) {
+                                             int tagP = -1, uint32_t epoch = 0) {
   // progress tags: (strip index << TAG_SHIFT) | columns done, monotonic per flag slot; the
   // strip index is the pass P, or the team stream's running strip index tagP (64-bit tags,
   // TAG_SHIFT = 32: the running index is unbounded and the query may have up to 2^20 columns)
@@ -348,6 +389,39 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
   auto fetch_group = [&](uint32_t (&rr)[4], uint32_t (&rh)[4], uint32_t (&rf)[4], int c0) {
 #pragma unroll
     for (int k = 0; k < 4; ++k) rr[k] = cols[min(c0 + k + 1, cmax)];
+    if constexpr (GPU_FLAGS) {
+      if (from_prev) {
+        const unsigned long long want = (unsigned long long)((epoch << 12) | (uint32_t)P) << 32;
+        const unsigned long long* q = reinterpret_cast<const unsigned long long*>(rb_in);
+        unsigned long long w[8];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const int i = min(c0 + k, rlast);
+          w[2 * k] = i < 0 ? want : ld_relaxed_gpu_u64(q + 2 * i);
+          w[2 * k + 1] = i < 0 ? want : ld_relaxed_gpu_u64(q + 2 * i + 1);
+        }
+        bool ready = true;
+#pragma unroll
+        for (int k = 0; k < 8; ++k) ready &= (w[k] & 0xffffffff00000000ull) == want;
+        while (!ready) {
+          __nanosleep(32);
+          ready = true;
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const int i = min(c0 + k, rlast);
+            if (i >= 0) {
+              w[2 * k] = ld_relaxed_gpu_u64(q + 2 * i);
+              w[2 * k + 1] = ld_relaxed_gpu_u64(q + 2 * i + 1);
+            }
+          }
+#pragma unroll
+          for (int k = 0; k < 8; ++k) ready &= (w[k] & 0xffffffff00000000ull) == want;
+        }
+#pragma unroll
+        for (int k = 0; k < 4; ++k) { rh[k] = (uint32_t)w[2 * k]; rf[k] = (uint32_t)w[2 * k + 1]; }
+      }
+      return;
+    }
     if (from_prev) {
       if constexpr (TEAM) {
         const TagT need = tag_prev | (TagT)(min(c0 + 3, rlast) + 1);
@@ -390,12 +464,21 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
       load_prof<R, CB, GC * CB>(wlo, prow + alo * ls);
     }
     uint32_t hup = x_hr, fs = x_f;
-    cell_rows<L, R, CC::kWide>(e, t, wlo, whi, nrho, prho, nsig, hup, fs, best, dlt);
+    cell_rows<L, R, CC::kWide, CHAIN2>(e, t, wlo, whi, nrho, prho, nsig, hup, fs, best, dlt);
     y_hr = hup; y_f = fs; y_res = x_res;
     // last lane: save the strip's bottom row for the next strip (not after the last strip);
     // fill steps write neutral values (index -1 keeps its neutral entry) that the real column
     // overwrites later.
-    if (store_out) rb_out[max(col, -1)] = make_uint2(y_hr, y_f);
+    if constexpr (GPU_FLAGS) {
+      if (store_out && col >= 0) {
+        const unsigned long long tg = (unsigned long long)((epoch << 12) | (uint32_t)(P + 1)) << 32;
+        unsigned long long* q = reinterpret_cast<unsigned long long*>(rb_out) + 2 * col;
+        st_relaxed_gpu_u64(q, tg | y_hr);
+        st_relaxed_gpu_u64(q + 1, tg | y_f);
+      }
+    } else if (store_out) {
+      rb_out[max(col, -1)] = make_uint2(y_hr, y_f);
+    }
     ++col;
   };
   // team mode: publish this strip's progress when a group crossed a multiple of PUB columns (16
@@ -404,7 +487,7 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
   // (short sweeps of the query: the next warp's wait is a larger share of each strip,
   // profiles/r01_pub_granularity.txt); team mode keeps 16.
   auto publish = [&]() {
-    if (TEAM && store_out) {
+    if (TEAM && !GPU_FLAGS && store_out) {
       const int done = col;   // the last lane's columns < col are stored
       if (done > 0 && (PUB == 4 || (done & 15) < 4 || done > rlast))
       {
@@ -1086,15 +1169,21 @@ __device__ __forceinline__ void t_gang_item(const TParams& p, const CC& c, uint8
   const int ncols = p.pair_ncols[gi];
   const int S = (ncols + LS - 1) / LS;
   const uint16_t* cp = p.cols + p.pair_off[gi];
-  uint2* rb = p.grb + (int64_t)gi * (GW + 1) * p.rb_cols;
-  uint32_t* prog = p.gprog + (int64_t)gi * (GW + 1);
+  // tagged hand-off slots: 2 uint2 (two 64-bit words) per column, slot s at 2 * s * rb_cols
+  uint2* rb = p.grb + (int64_t)gi * (GW + 1) * 2 * p.rb_cols;
   uint32_t b = 0;
   for (int P = gw; P < S; P += GW) {
     build_strip_tables<C>(p, tab, wp, cp, ncols, P);
     const int si = (P + GW) % (GW + 1), so = P % (GW + 1);
-    b = run_pass<L, 32, C, true, 16, true>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps, P, S,
-                                          rb + (int64_t)si * p.rb_cols + 1, rb + (int64_t)so * p.rb_cols + 1,
-                                          prog + si, prog + so, b);
+    uint2* in = rb + ((int64_t)si * p.rb_cols + 1) * 2;
+    uint2* out = rb + ((int64_t)so * p.rb_cols + 1) * 2;
+    if (p.gang_chain2)
+      b = run_pass<L, 32, C, true, 16, true, 20, false, true>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0,
+                                                              qsteps, P, S, in, out, (uint32_t*)nullptr,
+                                                              (uint32_t*)nullptr, b, -1, p.gang_epoch);
+    else
+      b = run_pass<L, 32, C, true, 16, true>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps, P, S, in,
+                                            out, (uint32_t*)nullptr, (uint32_t*)nullptr, b, -1, p.gang_epoch);
   }
 #pragma unroll
   for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));

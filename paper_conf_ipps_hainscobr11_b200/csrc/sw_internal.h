@@ -137,9 +137,11 @@ struct TParams {
   // gang_warps warps each; all buffers below are per gang pair and zeroed before the launch
   int gang_items, gang_ctas, gang_warps;
   int gang_share;            // 1: the gang CTAs' other warps run the team stream meanwhile
+  int gang_chain2;           // 1: the gang warps use the two-op vertical chain (cell_rows CHAIN2)
+  uint32_t gang_epoch;       // tag epoch of this launch's hand-off words (20 bits, != the last launch's)
   int32_t* gang_ctr;         // slot counter
-  uint32_t* gprog;           // gang_items x (GW + 1) progress flags, GW = gang_ctas * gang_warps
-  uint2* grb;                // gang_items x (GW + 1) x rb_cols row buffers
+  uint32_t* gprog;           // (unused: the hand-off words carry their own tags)
+  uint2* grb;                // gang_items x (GW + 1) x rb_cols x 2 tagged hand-off words (uint2 each)
   int32_t* gbest;            // gang_items x 2: maxima of the pair's two sequences
   int32_t* gdone;            // gang_items: warps finished
 };

@@ -109,10 +109,10 @@ def test_long_sequence_modes(mode, m):
         _assert_equal(out, ref, db, f"mode={mode} m={m} T={T}")
 
 
-@pytest.mark.parametrize("share", ["0", "1"])
+@pytest.mark.parametrize("variant", ["share0", "share1", "chain0"])
 @pytest.mark.parametrize("gang", ["2", "3", "8", "2:1", "5:3"])
 @pytest.mark.parametrize("m", [1, 144, 1500])
-def test_tmode_gangs(gang, m, share):
+def test_tmode_gangs(gang, m, variant):
     """T-mode gangs: the longest pairs spread over K CTAs (strip pipeline across CTAs through
     global row buffers and gpu-scope progress flags), SW_T_GANG = "K" (every long pair) or
     "K:items" (the items longest pairs); the other pairs take the CTA teams."""
@@ -123,9 +123,33 @@ def test_tmode_gangs(gang, m, share):
     q = gen.make_query(m, seed=990 + m)
     ref = _oracle(q, BLOSUM62, 10, 2, db)
     for T in (0, 3000):
-        out, _ = _gpu(q, BLOSUM62, 10, 2, db, T, env={"SW_LONG_MODE": "t", "SW_T_GANG": gang,
-                                                      "SW_T_GANG_SHARE": share})
-        _assert_equal(out, ref, db, f"gang={gang} m={m} T={T}")
+        env = {"SW_LONG_MODE": "t", "SW_T_GANG": gang, "SW_T_GANG_SHARE": "1" if variant == "share1" else "0",
+               "SW_T_GANG_CHAIN2": "0" if variant == "chain0" else "1"}
+        out, _ = _gpu(q, BLOSUM62, 10, 2, db, T, env=env)
+        _assert_equal(out, ref, db, f"gang={gang} m={m} T={T} {variant}")
+
+
+def test_tmode_gangs_repeated_searches():
+    """The gang hand-off words carry a per-launch epoch tag: repeated searches on one handle
+    (the same buffers, the same strip indices) must never read a word of an earlier launch."""
+    rng = np.random.default_rng(4)
+    lens = np.concatenate([[35213, 30000, 20000], rng.integers(3000, 9000, size=6)])
+    db = _db_from_lengths(lens, seed=61)
+    os.environ.update({"SW_LONG_MODE": "t", "SW_T_GANG": "4"})
+    try:
+        for m in (144, 567):
+            q = gen.make_query(m, seed=m + 1)
+            ref = _oracle(q, BLOSUM62, 10, 2, db)
+            with swp.SmithWaterman(q, BLOSUM62, 10, 2) as sw:
+                sw.load_db(db.residues, db.offsets)
+                for k in range(4):
+                    _assert_equal(sw.search(0), ref, db, f"m={m} repeat {k}")
+                outb = sw.search_batch([q, q, q], 0)
+                for k in range(3):
+                    _assert_equal(outb[k], ref, db, f"m={m} batch {k}")
+    finally:
+        os.environ.pop("SW_LONG_MODE", None)
+        os.environ.pop("SW_T_GANG", None)
 
 
 @pytest.mark.parametrize("team", [1, 2, 3, 5])
