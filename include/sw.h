@@ -160,6 +160,16 @@ int sw_last_stats(sw_handle h, int64_t out[4]);
  * Milliseconds. */
 int sw_last_kernel_ms(sw_handle h, double out[2]);
 
+/* Per-regime device time of the last search call (valid after its work completed), for the
+ * threshold sweeps (Fig.5 analog: share of the time in the intra-task kernel):
+ *   out[0] = sum over queries of the separate long-sequence launch (T-mode, on the query's
+ *            second stream, concurrent with the short-sequence launch; 0 when none ran),
+ *   out[1] = sum over queries of the whole search interval (== sw_last_kernel_ms out[0]),
+ *   out[2] = number of queries whose long sequences ran inside the fused search launch (team
+ *            mode, queries >= 3072 residues): their long-path time is part of out[1] only.
+ * Milliseconds (out[2]: a count). */
+int sw_last_regime_ms(sw_handle h, double out[3]);
+
 /* Optimal local alignment of the handle's query with database sequence seq_index (caller
  * order) — the traceback step after the search ("The optimal
  * alignment can be found by backtracking through H").  Computed on the device: an anti-

@@ -22,7 +22,7 @@ LIB_PATH = os.path.join(_HERE, "libsw_b200.so")
 SW_OK, SW_E_INVALID, SW_E_STATE, SW_E_NOMEM, SW_E_CUDA, SW_E_UNSUPPORTED = range(6)
 SW_AUTO_THRESHOLD = -1
 EXPORTED = ["sw_create", "sw_set_query", "sw_load_db", "sw_search", "sw_search_async",
-            "sw_search_batch", "sw_search_batch_async", "sw_search_stream", "sw_last_stats", "sw_last_kernel_ms", "sw_last_threshold",
+            "sw_search_batch", "sw_search_batch_async", "sw_search_stream", "sw_last_stats", "sw_last_kernel_ms", "sw_last_regime_ms", "sw_last_threshold",
             "sw_align", "sw_destroy",
             "sw_strerror", "sw_last_error", "sw_version"]
 
@@ -54,6 +54,7 @@ def load_library(path: str = LIB_PATH):
     L.sw_search_stream.argtypes = [vp, vp, vp, i32, vp, i64, vp, i64, vp, i32, i64]
     L.sw_last_stats.argtypes = [vp, vp]
     L.sw_last_kernel_ms.argtypes = [vp, vp]
+    L.sw_last_regime_ms.argtypes = [vp, vp]
     L.sw_last_threshold.argtypes = [vp]
     L.sw_align.argtypes = [vp, i64, vp, vp, i32]
     L.sw_align.restype = ctypes.c_int
@@ -66,7 +67,8 @@ def load_library(path: str = LIB_PATH):
     L.sw_last_error.restype = ctypes.c_char_p
     L.sw_version.restype = ctypes.c_char_p
     for name in ("sw_create", "sw_set_query", "sw_load_db", "sw_search", "sw_search_async", "sw_search_batch",
-                 "sw_search_batch_async", "sw_search_stream", "sw_last_stats", "sw_last_kernel_ms"):
+                 "sw_search_batch_async", "sw_search_stream", "sw_last_stats", "sw_last_kernel_ms",
+                 "sw_last_regime_ms"):
         getattr(L, name).restype = ctypes.c_int
     _lib = L
     return L
@@ -177,6 +179,12 @@ def sw_last_kernel_ms(h) -> dict:
     return {"search_ms": float(out[0]), "recompute_ms": float(out[1])}
 
 
+def sw_last_regime_ms(h) -> dict:
+    out = np.zeros(3, dtype=np.float64)
+    _check(h, load_library().sw_last_regime_ms(h, out.ctypes.data))
+    return {"long_ms": float(out[0]), "search_ms": float(out[1]), "fused_long_queries": int(out[2])}
+
+
 class Alignment(ctypes.Structure):
     _fields_ = [("score", ctypes.c_int32), ("q_begin", ctypes.c_int32), ("q_end", ctypes.c_int32),
                 ("d_begin", ctypes.c_int32), ("d_end", ctypes.c_int32), ("n_ops", ctypes.c_int32)]
@@ -236,6 +244,9 @@ class SmithWaterman:
 
     def kernel_ms(self) -> dict:
         return sw_last_kernel_ms(self.h)
+
+    def regime_ms(self) -> dict:
+        return sw_last_regime_ms(self.h)
 
     def align(self, seq_index: int) -> dict:
         return sw_align(self.h, seq_index)

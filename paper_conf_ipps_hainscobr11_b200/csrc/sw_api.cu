@@ -154,11 +154,16 @@ struct sw_handle_s {
   int stat_nq = 0;
   int32_t* h_ovf = nullptr;       // pinned, one overflow count per query of the last batch
   int h_ovf_cap = 0;
-  std::vector<cudaEvent_t> ev;    // 3 per query: before search, after search, after recompute
+  // kEvPerQuery per query: [0] before the search launches, [1] after them (long path joined),
+  // [2] after the recompute, [3] / [4] around the separate long-path (T-mode) launch
+  std::vector<cudaEvent_t> ev;
+  std::vector<char> long_fused;   // per query of the last batch: long pairs ran inside k_search
   std::string err;
 };
 
 namespace {
+
+constexpr int kEvPerQuery = 5;
 
 int fail(sw_handle h, int code, const std::string& msg) {
   if (h) h->err = msg;
@@ -639,6 +644,14 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
   p.rb_team = s.d_rb_team;
   p.rb_team_cols = max_cols_all;
   SW_CUDA(h, cudaEventRecord(ev[0], st));
+  {   // team mode: the long pairs run inside k_search (no separate long-path interval)
+    const size_t k = (size_t)(ev - h->ev.data()) / kEvPerQuery;
+    if (k < h->long_fused.size()) h->long_fused[k] = (char)(n_long > 0 && !use_t);
+  }
+  if (!use_t) {   // no separate long-path launch: an empty interval
+    SW_CUDA(h, cudaEventRecord(ev[3], st));
+    SW_CUDA(h, cudaEventRecord(ev[4], st));
+  }
   if (use_t) {
     // T-mode runs on the slot's second stream, concurrently with the group launch: its CTAs
     // take every SM first (launched first), and as they run out of long pairs the group
@@ -802,7 +815,9 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     t.rb_cols = qcols + kPadCols + 1;
     t.hi_mul = 1u << 24;
     if (t.gang_items > 0) SW_CUDA(h, cudaStreamWaitEvent(tst, h->gang_ev, 0));
+    SW_CUDA(h, cudaEventRecord(ev[3], tst));
     SW_CUDA(h, launch_tmode(t, t_grid, t_smem, tst));
+    SW_CUDA(h, cudaEventRecord(ev[4], tst));
     if (t.gang_items > 0) SW_CUDA(h, cudaEventRecord(h->gang_ev, tst));
     if (longq) {
       SW_CUDA(h, cudaEventRecord(ev[1], st));
@@ -1034,7 +1049,7 @@ int autotune(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq,
   // of the search launches, profile build to join, on the first slot)
   auto time_search = [&](int k, int32_t Tk, float* ms) -> int {
     const int m = (int)(qoff[k + 1] - qoff[k]);
-    cudaEvent_t* ev = h->ev.data() + 3 * k;
+    cudaEvent_t* ev = h->ev.data() + kEvPerQuery * k;
     int rc = enqueue_query(h, h->slots[0], d_queries + qoff[k], m, h->qmask[k], d_out + (int64_t)k * h->db->n_seqs,
                            Tk, h->h_ovf + k, ev);
     if (rc) return rc;
@@ -1133,7 +1148,8 @@ int run_batch(sw_handle h, const uint8_t* h_queries, const uint8_t* d_queries, c
     h->h_ovf_cap = nq;
   }
   memset(h->h_ovf, 0, (size_t)nq * sizeof(int32_t));
-  while ((int)h->ev.size() < 3 * nq) {
+  h->long_fused.assign((size_t)nq, 0);
+  while ((int)h->ev.size() < kEvPerQuery * nq) {
     cudaEvent_t e;
     SW_CUDA(h, cudaEventCreate(&e));
     h->ev.push_back(e);
@@ -1151,7 +1167,7 @@ int run_batch(sw_handle h, const uint8_t* h_queries, const uint8_t* d_queries, c
     QuerySlot& s = h->slots[k % ns];
     rc = enqueue_query(h, s, d_queries + qoff[k], (int)(qoff[k + 1] - qoff[k]), h->qmask[k],
                        d_out + (int64_t)k * h->db->n_seqs, T,
-                       h->h_ovf + k, h->ev.data() + 3 * k);
+                       h->h_ovf + k, h->ev.data() + kEvPerQuery * k);
     if (rc) return rc;
   }
   for (int k = 0; k < ns; ++k) {
@@ -1516,13 +1532,30 @@ int sw_align(sw_handle h, int64_t seq_index, sw_alignment* out, uint32_t* ops, i
 int sw_last_kernel_ms(sw_handle h, double out[2]) {
   if (!h || !out) return SW_E_INVALID;
   out[0] = out[1] = 0.0;
-  for (int k = 0; k < h->stat_nq && 3 * k + 2 < (int)h->ev.size(); ++k) {
+  for (int k = 0; k < h->stat_nq && kEvPerQuery * k + 2 < (int)h->ev.size(); ++k) {
     float a = 0.f, b = 0.f;
-    cudaError_t e = cudaEventElapsedTime(&a, h->ev[3 * k], h->ev[3 * k + 1]);
-    if (e == cudaSuccess) e = cudaEventElapsedTime(&b, h->ev[3 * k + 1], h->ev[3 * k + 2]);
+    const cudaEvent_t* ev = h->ev.data() + kEvPerQuery * k;
+    cudaError_t e = cudaEventElapsedTime(&a, ev[0], ev[1]);
+    if (e == cudaSuccess) e = cudaEventElapsedTime(&b, ev[1], ev[2]);
     if (e != cudaSuccess) return cuda_fail(h, e, "cudaEventElapsedTime");
     out[0] += a;
     out[1] += b;
+  }
+  return SW_OK;
+}
+
+int sw_last_regime_ms(sw_handle h, double out[3]) {
+  if (!h || !out) return SW_E_INVALID;
+  out[0] = out[1] = out[2] = 0.0;
+  for (int k = 0; k < h->stat_nq && kEvPerQuery * k + 4 < (int)h->ev.size(); ++k) {
+    float a = 0.f, b = 0.f;
+    const cudaEvent_t* ev = h->ev.data() + kEvPerQuery * k;
+    cudaError_t e = cudaEventElapsedTime(&a, ev[3], ev[4]);
+    if (e == cudaSuccess) e = cudaEventElapsedTime(&b, ev[0], ev[1]);
+    if (e != cudaSuccess) return cuda_fail(h, e, "cudaEventElapsedTime");
+    out[0] += a;
+    out[1] += b;
+    if (k < (int)h->long_fused.size() && h->long_fused[k]) out[2] += 1.0;
   }
   return SW_OK;
 }

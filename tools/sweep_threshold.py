@@ -34,6 +34,7 @@ def subset(mask):
 
 
 LAST_T = [None]
+LAST_REGIME = [None]
 
 
 def timed(res, off, T):
@@ -44,12 +45,14 @@ def timed(res, off, T):
         sw.search(T)
         sw.search(T)
         LAST_T[0] = sw.last_threshold()
+        LAST_REGIME[0] = sw.regime_ms()
         return sw.kernel_ms()["search_ms"]
 
 
 full_ms = {}
 for T in Ts:
     t_all = timed(db.residues, db.offsets, T)
+    reg = LAST_REGIME[0]
     auto = T < 0
     if auto:
         T = LAST_T[0]
@@ -61,7 +64,12 @@ for T in Ts:
             "frac_res_long": round(n_l / max(1, int(L.sum())), 5), "ms_total": round(t_all, 3),
             "gcups_total": round(m * int(L.sum()) / t_all / 1e6, 1) if t_all else None,
             "gcups_long_only": round(m * n_l / t_l / 1e6, 1) if t_l else None,
-            "gcups_short_only": round(m * n_s / t_s / 1e6, 1) if t_s else None}
+            "gcups_short_only": round(m * n_s / t_s / 1e6, 1) if t_s else None,
+            # Fig.5b analog: time of the long-path (T-mode) launch in the combined search, which
+            # runs concurrently with the short-sequence launch (share of the search interval)
+            "long_kernel_ms": round(reg["long_ms"], 3) if reg else None,
+            "pct_time_long_kernel": round(100 * reg["long_ms"] / reg["search_ms"], 1)
+            if reg and reg["search_ms"] > 0 and not reg["fused_long_queries"] else None}
     if line["gcups_long_only"] and line["gcups_short_only"]:
         line["long_over_short"] = round(line["gcups_long_only"] / line["gcups_short_only"], 3)
     print(json.dumps(line), flush=True)
