@@ -804,6 +804,12 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
       t.gang_epoch = h->gang_epoch;
       t.gang_chain2 = 1;
       if (const char* f = getenv("SW_T_GANG_CHAIN2")) t.gang_chain2 = atoi(f) != 0;
+      if (getenv("SW_DEBUG_GANG_TIMES")) {   // probe: per-strip times of gang item 0, printed below
+        static unsigned long long* d_dbg = nullptr;
+        if (!d_dbg) cudaMalloc(&d_dbg, 2 * 4096 * sizeof(unsigned long long));
+        cudaMemsetAsync(d_dbg, 0, 2 * 4096 * sizeof(unsigned long long), tst);
+        t.dbg_times = d_dbg;
+      }
       SW_CUDA(h, cudaMemsetAsync(s.d_gang, 0, ints * sizeof(int32_t), tst));
       t.gang_ctr = s.d_gang;
       t.gbest = s.d_gang + 1;
@@ -819,6 +825,16 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     SW_CUDA(h, launch_tmode(t, t_grid, t_smem, tst));
     SW_CUDA(h, cudaEventRecord(ev[4], tst));
     if (t.gang_items > 0) SW_CUDA(h, cudaEventRecord(h->gang_ev, tst));
+    if (t.dbg_times) {   // probe output: strip P start / end relative to strip 0's start (us)
+      std::vector<unsigned long long> tv(2 * 4096);
+      cudaStreamSynchronize(tst);
+      cudaMemcpy(tv.data(), t.dbg_times, tv.size() * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
+      const int S = (h->db->h_pair_ncols[0] + 32 * kTmodeC - 1) / (32 * kTmodeC);
+      fprintf(stderr, "gang item 0: %d strips, GW=%d, qsteps=%d\n", S, t.gang_ctas * t.gang_warps,
+              (int)round_up(qcols + 32, 4));
+      for (int P = 0; P < std::min(S, 4096); ++P)
+        fprintf(stderr, "strip %d start %.2f end %.2f us\n", P, (tv[2 * P] - tv[0]) / 1e3, (tv[2 * P + 1] - tv[0]) / 1e3);
+    }
     if (longq) {
       SW_CUDA(h, cudaEventRecord(ev[1], st));
       // exact 32-bit recompute of the flagged sequences: T-mode's LaneS32 instantiation (one

@@ -386,39 +386,44 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
   // group of 4 steps (lane-0 columns c0 .. c0 + 3), one team-mode wait per group: a
   // warp-uniform spin on a shared-memory flag (a divergent spin makes every later shuffle take
   // the slow diverged path).
+  // GPU_FLAGS: the tagged words of a group are loaded one group ahead (gload, with the
+  // residues) and their tags checked only when the group is about to run (gensure): the load
+  // latency hides behind a group of DP work and the wait is for the data the group needs
+  // (producer's column c0 + 3), not one group further
+  const unsigned long long want = (unsigned long long)((epoch << 12) | (uint32_t)P) << 32;
+  const unsigned long long* gq = reinterpret_cast<const unsigned long long*>(rb_in);
+  unsigned long long gA[8], gB[8];
+  int c0A = -1, c0B = -1;
+  auto gload = [&](unsigned long long (&g)[8], int c0) {
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const int i = min(c0 + k, rlast);
+      g[2 * k] = i < 0 ? want : ld_relaxed_gpu_u64(gq + 2 * i);
+      g[2 * k + 1] = i < 0 ? want : ld_relaxed_gpu_u64(gq + 2 * i + 1);
+    }
+  };
+  auto gensure = [&](unsigned long long (&g)[8], uint32_t (&rh)[4], uint32_t (&rf)[4], int c0) {
+    if (!from_prev) return;
+    bool ready = true;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) ready &= (g[k] & 0xffffffff00000000ull) == want;
+    while (!ready) {
+      __nanosleep(32);
+      gload(g, c0);
+      ready = true;
+#pragma unroll
+      for (int k = 0; k < 8; ++k) ready &= (g[k] & 0xffffffff00000000ull) == want;
+    }
+#pragma unroll
+    for (int k = 0; k < 4; ++k) { rh[k] = (uint32_t)g[2 * k]; rf[k] = (uint32_t)g[2 * k + 1]; }
+  };
   auto fetch_group = [&](uint32_t (&rr)[4], uint32_t (&rh)[4], uint32_t (&rf)[4], int c0) {
 #pragma unroll
     for (int k = 0; k < 4; ++k) rr[k] = cols[min(c0 + k + 1, cmax)];
     if constexpr (GPU_FLAGS) {
       if (from_prev) {
-        const unsigned long long want = (unsigned long long)((epoch << 12) | (uint32_t)P) << 32;
-        const unsigned long long* q = reinterpret_cast<const unsigned long long*>(rb_in);
-        unsigned long long w[8];
-#pragma unroll
-        for (int k = 0; k < 4; ++k) {
-          const int i = min(c0 + k, rlast);
-          w[2 * k] = i < 0 ? want : ld_relaxed_gpu_u64(q + 2 * i);
-          w[2 * k + 1] = i < 0 ? want : ld_relaxed_gpu_u64(q + 2 * i + 1);
-        }
-        bool ready = true;
-#pragma unroll
-        for (int k = 0; k < 8; ++k) ready &= (w[k] & 0xffffffff00000000ull) == want;
-        while (!ready) {
-          __nanosleep(32);
-          ready = true;
-#pragma unroll
-          for (int k = 0; k < 4; ++k) {
-            const int i = min(c0 + k, rlast);
-            if (i >= 0) {
-              w[2 * k] = ld_relaxed_gpu_u64(q + 2 * i);
-              w[2 * k + 1] = ld_relaxed_gpu_u64(q + 2 * i + 1);
-            }
-          }
-#pragma unroll
-          for (int k = 0; k < 8; ++k) ready &= (w[k] & 0xffffffff00000000ull) == want;
-        }
-#pragma unroll
-        for (int k = 0; k < 4; ++k) { rh[k] = (uint32_t)w[2 * k]; rf[k] = (uint32_t)w[2 * k + 1]; }
+        if (&rr == &rrA) { gload(gA, c0); c0A = c0; }
+        else { gload(gB, c0); c0B = c0; }
       }
       return;
     }
@@ -502,6 +507,7 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
   fetch_group(rrA, rhA, rfA, -1);
   for (int s = 0; s < steps; s += 8) {
     fetch_group(rrB, rhB, rfB, s + 3);
+    if constexpr (GPU_FLAGS) gensure(gA, rhA, rfA, c0A);
     step(std::integral_constant<int, 0>{}, rrA, rhA, rfA);
     step(std::integral_constant<int, 1>{}, rrA, rhA, rfA);
     step(std::integral_constant<int, 2>{}, rrA, rhA, rfA);
@@ -509,6 +515,7 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
     publish();
     if (s + 4 >= steps) break;
     fetch_group(rrA, rhA, rfA, s + 7);
+    if constexpr (GPU_FLAGS) gensure(gB, rhB, rfB, c0B);
     step(std::integral_constant<int, 0>{}, rrB, rhB, rfB);
     step(std::integral_constant<int, 1>{}, rrB, rhB, rfB);
     step(std::integral_constant<int, 2>{}, rrB, rhB, rfB);
@@ -1174,6 +1181,11 @@ __device__ __forceinline__ void t_gang_item(const TParams& p, const CC& c, uint8
   uint32_t b = 0;
   for (int P = gw; P < S; P += GW) {
     build_strip_tables<C>(p, tab, wp, cp, ncols, P);
+    if (p.dbg_times && gi == 0 && lane == 0 && P < 4096) {   // probe: strip start (ns)
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      p.dbg_times[2 * P] = t;
+    }
     const int si = (P + GW) % (GW + 1), so = P % (GW + 1);
     uint2* in = rb + ((int64_t)si * p.rb_cols + 1) * 2;
     uint2* out = rb + ((int64_t)so * p.rb_cols + 1) * 2;
@@ -1184,6 +1196,11 @@ __device__ __forceinline__ void t_gang_item(const TParams& p, const CC& c, uint8
     else
       b = run_pass<L, 32, C, true, 16, true>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps, P, S, in,
                                             out, (uint32_t*)nullptr, (uint32_t*)nullptr, b, -1, p.gang_epoch);
+    if (p.dbg_times && gi == 0 && lane == 0 && P < 4096) {   // probe: strip end (ns)
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      p.dbg_times[2 * P + 1] = t;
+    }
   }
 #pragma unroll
   for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));

@@ -139,6 +139,7 @@ struct TParams {
   int gang_share;            // 1: the gang CTAs' other warps run the team stream meanwhile
   int gang_chain2;           // 1: the gang warps use the two-op vertical chain (cell_rows CHAIN2)
   uint32_t gang_epoch;       // tag epoch of this launch's hand-off words (20 bits, != the last launch's)
+  unsigned long long* dbg_times;   // probe (SW_DEBUG_GANG_TIMES): gang item 0's strip start / end (ns)
   int32_t* gang_ctr;         // slot counter
   uint32_t* gprog;           // (unused: the hand-off words carry their own tags)
   uint2* grb;                // gang_items x (GW + 1) x rb_cols x 2 tagged hand-off words (uint2 each)
