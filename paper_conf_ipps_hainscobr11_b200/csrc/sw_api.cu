@@ -753,13 +753,23 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
         const bool hidden = (double)sp.short_cols > 0.5 * (double)sp.long_cols;
         int K = 0, items = 0;
         if (!hidden) {
+          // a gang of GW warps: each warp runs ceil(S / GW) strips back to back after a ramp of
+          // (GW - 1) lags, unless the wavefront (S - 1) lag + qsteps is longer (measured per
+          // strip with SW_DEBUG_GANG_TIMES: the C2 35,213-residue pair, query 567: 3 CTAs
+          // 0.81 ms, 4-8 CTAs 0.72 ms, profiles/r02_gang_*.txt)
+          auto gang_time = [&](int GW, double S) {
+            return std::max(std::ceil(S / GW) * qsteps + (std::min<double>(GW, S) - 1.0) * lag,
+                            (S - 1.0) * lag + qsteps);
+          };
           for (int pp = 0; pp < n_long && pp < kMaxGangItems; ++pp) {
             const double S = std::ceil((double)h->db->h_pair_ncols[pp] / spos);
             const double alone = item_time(S >= t.big_strips ? t_warps : W, S);
             if (alone <= 1.15 * t_thr || S < 2.0 * W) break;
-            const double goal = std::max(1.15 * t_thr, 1.05 * ((S - 1.0) * lag + qsteps));
+            double best_g = 1e300;
+            for (int k = 2; k <= kMaxGangCtas; ++k) best_g = std::min(best_g, gang_time(k * WG, S));
+            const double goal = std::max(1.15 * t_thr, 1.03 * best_g);
             int k = 2;
-            while (k < kMaxGangCtas && item_time(k * WG, S) > goal) ++k;
+            while (k < kMaxGangCtas && gang_time(k * WG, S) > goal) ++k;
             K = std::max(K, k);
             ++items;
           }
@@ -771,6 +781,9 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
           items = comma ? atoi(comma + 1) : n_long;
           items = std::min(items, std::min(n_long, t_grid / std::max(1, K)));
         }
+        // the 4-bit hand-off tags (run_pass GPU_FLAGS) repeat every 15 strips: a slot is reused
+        // every GW + 1 strips, which must not be a multiple of 15
+        while (K >= 2 && (K * WG + 1) % 15 == 0) --K;
         if (getenv("SW_DEBUG_PLAN"))
           fprintf(stderr, "tmode m=%d long_pairs=%d W=%d t_warps=%d big=%d thr=%.0f steps gangs=%d x %d CTAs\n", m,
                   n_long, W, t_warps, t.big_strips, t_thr, items, K);
@@ -791,17 +804,12 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
       const size_t ints = 1 + 3 * (size_t)t.gang_items + (size_t)t.gang_items * (GW + 1);
       rc = grow(h, &s.d_gang, &s.gang_cap, ints * sizeof(int32_t), "alloc gang scratch", tst);
       if (rc) return rc;
-      const size_t grb_bytes = (size_t)t.gang_items * (GW + 1) * (qcols + kPadCols + 1) * 2 * sizeof(uint2);
+      const size_t grb_bytes = (size_t)t.gang_items * (GW + 1) * (qcols + kPadCols + 1) * sizeof(uint2);
       rc = grow(h, &s.d_grb, &s.grb_cap, grb_bytes, "alloc gang row buffers", tst, true);
       if (rc) return rc;
-      // hand-off words are tagged with a launch epoch: a word left by an earlier launch never
-      // matches (cleared when the 20-bit epoch wraps)
-      h->gang_epoch = (h->gang_epoch + 1) & 0xfffff;
-      if (h->gang_epoch == 0) {
-        SW_CUDA(h, cudaMemsetAsync(s.d_grb, 0, s.grb_cap, tst));
-        h->gang_epoch = 1;
-      }
-      t.gang_epoch = h->gang_epoch;
+      // the hand-off words carry a 4-bit strip tag (never 0): clear what an earlier launch left
+      SW_CUDA(h, cudaMemsetAsync(s.d_grb, 0, grb_bytes, tst));
+      t.gang_epoch = 0;
       t.gang_chain2 = 1;
       if (const char* f = getenv("SW_T_GANG_CHAIN2")) t.gang_chain2 = atoi(f) != 0;
       if (getenv("SW_DEBUG_GANG_TIMES")) {   // probe: per-strip times of gang item 0, printed below

@@ -328,11 +328,15 @@ __device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&t)[R], co
 // neutral fill values).  Returns max(best, this lane's H maxima) (packed per Lane).
 // ONE_PASS: the query is one strip (no row buffer in or out): the first lane's top input is
 // the constant boundary (0, 0), so the boundary rings and their loads disappear (registers).
-// GPU_FLAGS (T-mode gangs, strips on different SMs): the row buffers hold two tagged 64-bit
-// words per column, (tag << 32 | H) and (tag << 32 | F + rho) with tag = epoch << 12 | (P + 1),
-// written by the producing strip's last lane as it goes; the consuming strip's lane 0 polls
-// the words it needs (a per-column "flag in the data": no release fence, no progress flag,
-// no publication granularity).  prog_in / prog_out are unused then.
+// GPU_FLAGS (T-mode gangs, strips on different SMs): the row buffers hold ONE tagged 64-bit word
+// per column, H | (F + rho) << 32, whose four s16 halves carry a 4-bit tag in their bit 15:
+// every half is in [0, 32767) for a sequence that is not flagged (H >= 0, F + rho >= 0, both
+// below the overflow flag), and a flagged sequence's values are recomputed anyway.  The
+// producing strip's last lane writes the words as it goes; the consuming strip's lane 0 polls
+// the words it needs (a per-column "flag in the data": no release fence, no progress flag, no
+// publication granularity).  tag = 1 + P mod 15 (never 0, the cleared buffer), and slot reuse
+// every GW + 1 strips changes it (the planner keeps (GW + 1) mod 15 != 0); the buffer is
+// cleared before every gang launch.  prog_in / prog_out are unused then.
 template <class L, int GC, int R, bool TEAM, int PUB = 16, bool GPU_FLAGS = false, int TAG_SHIFT = 20,
           bool ONE_PASS = false, bool CHAIN2 = false, class CC = ChainConst, class TagT = uint32_t>
 __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, int ls, int hi_off,
@@ -386,47 +390,53 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
   // group of 4 steps (lane-0 columns c0 .. c0 + 3), one team-mode wait per group: a
   // warp-uniform spin on a shared-memory flag (a divergent spin makes every later shuffle take
   // the slow diverged path).
-  // GPU_FLAGS: the tagged words of a group are loaded one group ahead (gload, with the
-  // residues) and their tags checked only when the group is about to run (gensure): the load
-  // latency hides behind a group of DP work and the wait is for the data the group needs
-  // (producer's column c0 + 3), not one group further
-  const unsigned long long want = (unsigned long long)((epoch << 12) | (uint32_t)P) << 32;
+  // GPU_FLAGS: the tagged words of a group are loaded two groups ahead (gload right after
+  // the ring's previous group was checked and unpacked) and their tags are checked only when
+  // the group is about to run (gensure): the load latency hides behind two groups of DP work,
+  // and the wait is for the data the group needs (the producer's column c0 + 3)
+  constexpr unsigned long long kTagBits = 0x8000800080008000ull;
+  auto tag_bits = [](uint32_t tg) -> unsigned long long {   // 4-bit tag -> bit 15 of each half
+    return ((unsigned long long)(tg & 1) << 15) | ((unsigned long long)((tg >> 1) & 1) << 31) |
+           ((unsigned long long)((tg >> 2) & 1) << 47) | ((unsigned long long)((tg >> 3) & 1) << 63);
+  };
+  const unsigned long long want = tag_bits(1u + (uint32_t)(P + 14) % 15u);   // strip P - 1's tag
+  const unsigned long long mine = tag_bits(1u + (uint32_t)P % 15u);
   const unsigned long long* gq = reinterpret_cast<const unsigned long long*>(rb_in);
-  unsigned long long gA[8], gB[8];
-  int c0A = -1, c0B = -1;
-  auto gload = [&](unsigned long long (&g)[8], int c0) {
+  unsigned long long gA[4], gB[4];
+  int c0A = -1, c0B = 3;
+  auto gload = [&](unsigned long long (&g)[4], int c0) {
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
       const int i = min(c0 + k, rlast);
-      g[2 * k] = i < 0 ? want : ld_relaxed_gpu_u64(gq + 2 * i);
-      g[2 * k + 1] = i < 0 ? want : ld_relaxed_gpu_u64(gq + 2 * i + 1);
+      g[k] = i < 0 ? want : ld_relaxed_gpu_u64(gq + i);
     }
   };
-  auto gensure = [&](unsigned long long (&g)[8], uint32_t (&rh)[4], uint32_t (&rf)[4], int c0) {
-    if (!from_prev) return;
+  auto gensure = [&](unsigned long long (&g)[4], uint32_t (&rh)[4], uint32_t (&rf)[4], int& c0) {
     bool ready = true;
 #pragma unroll
-    for (int k = 0; k < 8; ++k) ready &= (g[k] & 0xffffffff00000000ull) == want;
+    for (int k = 0; k < 4; ++k) ready &= (g[k] & kTagBits) == want;
     while (!ready) {
       __nanosleep(32);
       gload(g, c0);
       ready = true;
 #pragma unroll
-      for (int k = 0; k < 8; ++k) ready &= (g[k] & 0xffffffff00000000ull) == want;
+      for (int k = 0; k < 4; ++k) ready &= (g[k] & kTagBits) == want;
     }
 #pragma unroll
-    for (int k = 0; k < 4; ++k) { rh[k] = (uint32_t)g[2 * k]; rf[k] = (uint32_t)g[2 * k + 1]; }
+    for (int k = 0; k < 4; ++k) {
+      const unsigned long long v = g[k] & ~kTagBits;
+      rh[k] = (uint32_t)v; rf[k] = (uint32_t)(v >> 32);
+    }
+    c0 += 8;
+    gload(g, c0);   // the ring's next group (two groups ahead)
   };
+  if constexpr (GPU_FLAGS) {
+    if (from_prev) { gload(gA, c0A); gload(gB, c0B); }
+  }
   auto fetch_group = [&](uint32_t (&rr)[4], uint32_t (&rh)[4], uint32_t (&rf)[4], int c0) {
 #pragma unroll
     for (int k = 0; k < 4; ++k) rr[k] = cols[min(c0 + k + 1, cmax)];
-    if constexpr (GPU_FLAGS) {
-      if (from_prev) {
-        if (&rr == &rrA) { gload(gA, c0); c0A = c0; }
-        else { gload(gB, c0); c0B = c0; }
-      }
-      return;
-    }
+    if constexpr (GPU_FLAGS) return;
     if (from_prev) {
       if constexpr (TEAM) {
         const TagT need = tag_prev | (TagT)(min(c0 + 3, rlast) + 1);
@@ -476,10 +486,8 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
     // overwrites later.
     if constexpr (GPU_FLAGS) {
       if (store_out && col >= 0) {
-        const unsigned long long tg = (unsigned long long)((epoch << 12) | (uint32_t)(P + 1)) << 32;
-        unsigned long long* q = reinterpret_cast<unsigned long long*>(rb_out) + 2 * col;
-        st_relaxed_gpu_u64(q, tg | y_hr);
-        st_relaxed_gpu_u64(q + 1, tg | y_f);
+        const unsigned long long v = ((unsigned long long)y_f << 32 | y_hr) & ~kTagBits;
+        st_relaxed_gpu_u64(reinterpret_cast<unsigned long long*>(rb_out) + col, v | mine);
       }
     } else if (store_out) {
       rb_out[max(col, -1)] = make_uint2(y_hr, y_f);
@@ -507,7 +515,7 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
   fetch_group(rrA, rhA, rfA, -1);
   for (int s = 0; s < steps; s += 8) {
     fetch_group(rrB, rhB, rfB, s + 3);
-    if constexpr (GPU_FLAGS) gensure(gA, rhA, rfA, c0A);
+    if constexpr (GPU_FLAGS) { if (from_prev) gensure(gA, rhA, rfA, c0A); }
     step(std::integral_constant<int, 0>{}, rrA, rhA, rfA);
     step(std::integral_constant<int, 1>{}, rrA, rhA, rfA);
     step(std::integral_constant<int, 2>{}, rrA, rhA, rfA);
@@ -515,7 +523,7 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
     publish();
     if (s + 4 >= steps) break;
     fetch_group(rrA, rhA, rfA, s + 7);
-    if constexpr (GPU_FLAGS) gensure(gB, rhB, rfB, c0B);
+    if constexpr (GPU_FLAGS) { if (from_prev) gensure(gB, rhB, rfB, c0B); }
     step(std::integral_constant<int, 0>{}, rrB, rhB, rfB);
     step(std::integral_constant<int, 1>{}, rrB, rhB, rfB);
     step(std::integral_constant<int, 2>{}, rrB, rhB, rfB);
@@ -1176,8 +1184,8 @@ __device__ __forceinline__ void t_gang_item(const TParams& p, const CC& c, uint8
   const int ncols = p.pair_ncols[gi];
   const int S = (ncols + LS - 1) / LS;
   const uint16_t* cp = p.cols + p.pair_off[gi];
-  // tagged hand-off slots: 2 uint2 (two 64-bit words) per column, slot s at 2 * s * rb_cols
-  uint2* rb = p.grb + (int64_t)gi * (GW + 1) * 2 * p.rb_cols;
+  // tagged hand-off slots: one 64-bit word per column (run_pass GPU_FLAGS)
+  uint2* rb = p.grb + (int64_t)gi * (GW + 1) * p.rb_cols;
   uint32_t b = 0;
   for (int P = gw; P < S; P += GW) {
     build_strip_tables<C>(p, tab, wp, cp, ncols, P);
@@ -1187,8 +1195,8 @@ __device__ __forceinline__ void t_gang_item(const TParams& p, const CC& c, uint8
       p.dbg_times[2 * P] = t;
     }
     const int si = (P + GW) % (GW + 1), so = P % (GW + 1);
-    uint2* in = rb + ((int64_t)si * p.rb_cols + 1) * 2;
-    uint2* out = rb + ((int64_t)so * p.rb_cols + 1) * 2;
+    uint2* in = rb + (int64_t)si * p.rb_cols + 1;
+    uint2* out = rb + (int64_t)so * p.rb_cols + 1;
     if (p.gang_chain2)
       b = run_pass<L, 32, C, true, 16, true, 20, false, true>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0,
                                                               qsteps, P, S, in, out, (uint32_t*)nullptr,
