@@ -118,7 +118,7 @@ int sw_search_batch_async(sw_handle h, const uint8_t* queries, const int64_t* q_
  * the planner's 5 best kernel configurations, one search each, on the handle's first internal
  * stream, and keeps the fastest for later searches of that (query length, threshold).  With
  * length_threshold == SW_AUTO_THRESHOLD the first search of a query length with >= 1e9 cells
- * also times the threshold model's two best candidates and the all-short endpoint (plus the
+ * also times the threshold model's four best candidates and the all-short endpoint (plus the
  * all-long one on databases whose sequences are all >= 512) and keeps the fastest threshold
  * for that query length.  That first call therefore synchronises with the device (the async
  * variants block for it) and costs a few searches; its scores are the exact ones (every

@@ -581,7 +581,9 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
   const int a_used = __builtin_popcount(qmask);
   const int wp_bytes = (int)round_up((int64_t)(a_used + 1) * kWpStride, 128);
   const int per_warp = 2 * (a_used + 1) * 32 * kTmodeC;
-  int t_warps = std::min(kTmodeThreads / 32, (kMaxProfileSmem - wp_bytes) / per_warp);
+  // (k_search_t also holds ~19 KB of static shared memory: the team streams' pair rings)
+  constexpr int kTmodeSmemBudget = (227 - 20) * 1024;
+  int t_warps = std::min(kTmodeThreads / 32, (kTmodeSmemBudget - wp_bytes) / per_warp);
   if (t_warps < 1) use_t = false;
   int t_grid = 0;
   const int t_smem = wp_bytes + t_warps * per_warp;
@@ -1087,14 +1089,14 @@ int autotune(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq,
     // Automatic threshold: the model's estimate misses the occupancy of group
     // launches with few items and the long path's tail, by up to 4x on long-sequence databases
     // (C3 query 144).  The first search of a query length with
-    // SW_AUTO_THRESHOLD on a loaded database of >= kTuneTMinCells cells times the model's two
+    // SW_AUTO_THRESHOLD on a loaded database of >= kTuneTMinCells cells times the model's four
     // best thresholds and the endpoints (all short: T > max length; all long: T = min length,
     // for long-sequence databases) and keeps the fastest.
     if (T == SW_AUTO_THRESHOLD && (double)m * residues >= kTuneTMinCells && !h->tuned_T.count(m)) {
       const auto ranked = rank_thresholds(h, m);
       std::vector<int64_t> cand;
-      for (const auto& c : ranked) {
-        if ((int)cand.size() >= 2) break;
+      for (const auto& c : ranked) {   // (the model's ranking is off by up to ~10 % between
+        if ((int)cand.size() >= 4) break;   // neighbouring candidates: profiles/r02_variance_sweep)
         cand.push_back(c.second);
       }
       const int64_t all_short = h->db->sorted_len.empty() ? 0 : h->db->sorted_len[0] + 1;

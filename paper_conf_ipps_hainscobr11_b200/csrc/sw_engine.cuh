@@ -337,6 +337,8 @@ __device__ __forceinline__ void cell_rows(uint32_t (&e)[R], uint32_t (&t)[R], co
 // publication granularity).  tag = 1 + P mod 15 (never 0, the cleared buffer), and slot reuse
 // every GW + 1 strips changes it (the planner keeps (GW + 1) mod 15 != 0); the buffer is
 // cleared before every gang launch.  prog_in / prog_out are unused then.
+// keep (the packed T-mode team stream): 0 for a lane whose rows start a new database pair —
+// its vertical input (the lane above's bottom row) is replaced by the neutral boundary.
 template <class L, int GC, int R, bool TEAM, int PUB = 16, bool GPU_FLAGS = false, int TAG_SHIFT = 20,
           bool ONE_PASS = false, bool CHAIN2 = false, class CC = ChainConst, class TagT = uint32_t>
 __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, int ls, int hi_off,
@@ -344,7 +346,7 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
                                              int half, int steps, int P, int passes_total,
                                              const uint2* __restrict__ rb_in, uint2* __restrict__ rb_out,
                                              const TagT* prog_in, TagT* prog_out, uint32_t best,
-                                             int tagP = -1, uint32_t epoch = 0) {
+                                             int tagP = -1, uint32_t epoch = 0, uint32_t keep = 1u) {
   // progress tags: (strip index << TAG_SHIFT) | columns done, monotonic per flag slot; the
   // strip index is the pass P, or the team stream's running strip index tagP (64-bit tags,
   // TAG_SHIFT = 32: the running index is unbounded and the query may have up to 2^20 columns)
@@ -465,6 +467,7 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
       if (gl == 0) x_res = rr[K];
     } else {
       if (gl == 0) { x_hr = rh[K]; x_f = rf[K]; x_res = rr[K]; }
+      if constexpr (TAG_SHIFT == 32) { x_hr *= keep; x_f *= keep; }   // (IMAD) packed team stream
     }
     // query-profile words for the two letters of the NEXT column (look-ahead u)
     uint32_t wlo[(R + 3) / 4], whi[(R + 3) / 4];
@@ -925,9 +928,11 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
 // P_lo[a][pos] = w(a, d_lo[pos]) + rho (a = compact query letter), P_hi likewise, chunk-major
 // and lane-private like the query profile (every lane writes and later reads only its chunks).
 // SEQS = 1 (32-bit recompute of one flagged sequence): only P_lo, for the pair's half-th sequence.
+// pos0: the lane's first database position (P * 32C + lane * C for the strips of one pair; in
+// the packed team stream every lane has its own pair, cp and position); ncols <= 0: pad lane.
 template <int C, int SEQS = 2>
 __device__ __forceinline__ void build_strip_tables(const TParams& p, uint8_t* tab, const int8_t* wp,
-                                                   const uint16_t* cp, int ncols, int P, int half = 0) {
+                                                   const uint16_t* cp, int ncols, int pos0, int half = 0) {
   constexpr int CB = chunk_bytes<C>();
   constexpr int LS = 32 * C;
   const int lane = threadIdx.x & 31;
@@ -937,7 +942,7 @@ __device__ __forceinline__ void build_strip_tables(const TParams& p, uint8_t* ta
   uint32_t dp[C];
 #pragma unroll
   for (int r = 0; r < C; ++r) {
-    const int pos = P * LS + lane * C + r;
+    const int pos = pos0 + r;
     dp[r] = pos < ncols ? (uint32_t)cp[pos] : db_pad;
   }
   for (int a = 0; a < A1; ++a) {
@@ -1015,7 +1020,7 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const CC& c, uint8
     const uint16_t* cp = p.cols + p.pair_off[item];
     uint32_t b = 0;
     for (int P = wt; P < S; P += W) {
-      build_strip_tables<C>(p, tab, wp, cp, ncols, P);
+      build_strip_tables<C>(p, tab, wp, cp, ncols, P * LS + lane * C);
       const int si = (P + W) % (W + 1), so = P % (W + 1);
       b = run_pass<L, 32, C, true, 4>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps, P, S,
                                      rb + (int64_t)si * p.rb_cols + 1, rb + (int64_t)so * p.rb_cols + 1, prog + si,
@@ -1042,10 +1047,18 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const CC& c, uint8
 // (slot g mod (W + 1), tag = g): strip g + 1 consumes strip g's bottom row only inside a pair.
 // Each pair's maximum is combined with atomicMax in the team's shared ring of pairs; the
 // warp finishing its last strip emits the scores.
-constexpr int kTQ = 16;      // pairs in a team's ring (a team spans at most ~W + 1 of them)
+// PACKED: the team's pairs are laid out back to back in LANES of C database positions (a pair
+// of n' columns takes ceil(n' / C) lanes) and strip g is the team's lanes [32g, 32g + 32): a
+// strip holds the tail of one pair and the heads of the next ones, so short pairs no longer
+// leave most of a 32-lane strip idle (a 350-column pair used 22 of 32 lanes).  A lane whose rows
+// start a pair takes the neutral boundary instead of the lane above's bottom row (run_pass
+// keep), strip g + 1 takes strip g's bottom row only when its first lane continues a pair, and
+// every lane folds its maximum into its pair's entry (atomicMax in shared memory); the lane
+// that completes a pair's last lane emits its scores.
+constexpr int kTQ = 96;      // pairs in a team's ring: W strips x 32 lanes / >= 3 lanes per pair
 struct TStream {
-  int lock, count, next, end;
-  int item[kTQ], base[kTQ], S[kTQ], rem[kTQ], mlo[kTQ], mhi[kTQ];
+  int lock, count, next, end;   // next: lanes appended so far
+  int item[kTQ], base[kTQ], nl[kTQ], rem[kTQ], mlo[kTQ], mhi[kTQ];
 };
 
 // L = LaneS32: the 32-bit recompute of the flagged sequences (items = positions of
@@ -1078,18 +1091,17 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
     if constexpr (S32) emit_t32(p, lo, p.item_list[item]);
     else emit_t(p, ((uint32_t)lo & 0xffffu) | ((uint32_t)hi << 16), item);
   };
-  // append one pair to the ring (lane 0 of the warp holding the lock); empty pairs score 0
+  // append one pair to the ring (lane 0 of the warp holding the lock)
   auto append = [&](int item) {
     int hf;
-    const int S = (p.pair_ncols[pair_of(item, &hf)] + LS - 1) / LS;
-    if (S == 0) { emit_item(item, 0, 0); return; }
+    const int nl = (p.pair_ncols[pair_of(item, &hf)] + C - 1) / C;   // >= 3 lanes (n' >= 48)
     const int k = vs->count % kTQ;
     if (vs->count >= kTQ)   // the entry kTQ pairs back must be finished before it is reused
       while (vs->rem[k] != 0) __nanosleep(64);
-    vs->item[k] = item; vs->base[k] = vs->next; vs->S[k] = S; vs->rem[k] = S; vs->mlo[k] = 0; vs->mhi[k] = 0;
+    vs->item[k] = item; vs->base[k] = vs->next; vs->nl[k] = nl; vs->rem[k] = nl; vs->mlo[k] = 0; vs->mhi[k] = 0;
     __threadfence_block();
     vs->count = vs->count + 1;
-    vs->next = vs->next + S;
+    vs->next = vs->next + nl;
   };
   team_bar(team, W);
   if (wt == 0 && lane == 0) {
@@ -1100,21 +1112,13 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
   }
   team_bar(team, W);
   for (int g = wt;; g += W) {
-    // the ring entry of strip g (lane 0 decides, the warp follows)
-    int k = -1;
+    // strip g needs every pair that covers its lanes (lane 0 appends, the warp follows)
+    int have = 0;
     if (lane == 0) {
       for (;;) {
-        const int next = vs->next, count = vs->count;
-        if (g < next) {
-          for (int j = count - 1; j >= 0 && j >= count - kTQ; --j) {
-            const int kk = j % kTQ;
-            if (vs->base[kk] <= g) { k = kk; break; }
-          }
-          break;
-        }
-        if (vs->end) break;
+        if (vs->next >= 32 * g + 32 || vs->end) { have = vs->next > 32 * g; break; }
         if (atomicCAS(&ts->lock, 0, 1) == 0) {
-          while (vs->next <= g && !vs->end) {
+          while (vs->next < 32 * g + 32 && !vs->end) {
             const int item = p.gang_items + atomicAdd(p.work, 1);
             if (item >= n_items) { vs->end = 1; break; }
             append(item);
@@ -1126,21 +1130,36 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
         }
       }
     }
-    k = __shfl_sync(SWB_FULL, k, 0);
-    if (k < 0) break;
-    const int item = vs->item[k], P = g - vs->base[k], S = vs->S[k];
-    int half;
-    const int pair = pair_of(item, &half);
-    const int ncols = p.pair_ncols[pair];
-    const uint16_t* cp = p.cols + p.pair_off[pair];
-    build_strip_tables<C, L::kSeqs>(p, tab, wp, cp, ncols, P, half);
+    have = __shfl_sync(SWB_FULL, have, 0);
+    if (!have) break;
+    // this lane's pair: the newest ring entry starting at or before lane 32g + lane
+    const int gl = 32 * g + lane;
+    int k = -1;
+    {
+      const int count = vs->count;
+      for (int j = count - 1; j >= 0 && j >= count - kTQ; --j) {
+        const int kk = j % kTQ;
+        if (vs->base[kk] <= gl) { if (gl < vs->base[kk] + vs->nl[kk]) k = kk; break; }
+      }
+    }
+    int item = -1, half = 0, pair = 0, ncols = 0, lip = 0;
+    if (k >= 0) {
+      item = vs->item[k];
+      pair = pair_of(item, &half);
+      ncols = p.pair_ncols[pair];
+      lip = gl - vs->base[k];             // lane index within the pair
+    }
+    const uint16_t* cp = p.cols + (k >= 0 ? p.pair_off[pair] : 0);
+    build_strip_tables<C, L::kSeqs>(p, tab, wp, cp, k >= 0 ? ncols : 0, lip * C, half);
+    // strip g continues strip g - 1's pair in its first lane: take its bottom row
+    const int cont = __shfl_sync(SWB_FULL, k >= 0 && lip > 0 ? 1 : 0, 0);
+    const uint32_t keep = (lane > 0 && k >= 0 && lip == 0) ? 0u : 1u;
     const int si = (g + W) % (W + 1), so = g % (W + 1);
     uint32_t b = run_pass<L, 32, C, true, 4, false, 32>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps,
-                                                       P, S, rb + (int64_t)si * p.rb_cols + 1,
-                                                       rb + (int64_t)so * p.rb_cols + 1, prog + si, prog + so, 0u, g);
-#pragma unroll
-    for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
-    if (lane == 0) {
+                                                       cont, 3, rb + (int64_t)si * p.rb_cols + 1,
+                                                       rb + (int64_t)so * p.rb_cols + 1, prog + si, prog + so, 0u, g,
+                                                       0u, keep);
+    if (k >= 0) {
       if constexpr (S32) {
         atomicMax(&ts->mlo[k], (int)b);
       } else {
@@ -1148,7 +1167,7 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
         atomicMax(&ts->mhi[k], (int)(int16_t)(b >> 16));
       }
       __threadfence_block();
-      if (atomicSub(&ts->rem[k], 1) == 1) {   // this pair's last strip
+      if (atomicSub(&ts->rem[k], 1) == 1) {   // this pair's last lane
         const int lo = atomicAdd(&ts->mlo[k], 0), hi = atomicAdd(&ts->mhi[k], 0);
         emit_item(item, lo, hi);
       }
@@ -1188,7 +1207,7 @@ __device__ __forceinline__ void t_gang_item(const TParams& p, const CC& c, uint8
   uint2* rb = p.grb + (int64_t)gi * (GW + 1) * p.rb_cols;
   uint32_t b = 0;
   for (int P = gw; P < S; P += GW) {
-    build_strip_tables<C>(p, tab, wp, cp, ncols, P);
+    build_strip_tables<C>(p, tab, wp, cp, ncols, P * LS + lane * C);
     if (p.dbg_times && gi == 0 && lane == 0 && P < 4096) {   // probe: strip start (ns)
       unsigned long long t;
       asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
