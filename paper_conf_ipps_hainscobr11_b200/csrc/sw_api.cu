@@ -581,9 +581,9 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
   const int a_used = __builtin_popcount(qmask);
   const int wp_bytes = (int)round_up((int64_t)(a_used + 1) * kWpStride, 128);
   const int per_warp = 2 * (a_used + 1) * 32 * kTmodeC;
-  // (k_search_t also holds ~19 KB of static shared memory: the team streams' pair rings)
-  constexpr int kTmodeSmemBudget = (227 - 20) * 1024;
-  int t_warps = std::min(kTmodeThreads / 32, (kTmodeSmemBudget - wp_bytes) / per_warp);
+  // (k_search_t also holds ~3 KB of static shared memory: progress flags, the team streams' pair
+  // pool; 220 KB + 3 KB stays below the 227 KB per CTA)
+  int t_warps = std::min(kTmodeThreads / 32, (kMaxProfileSmem - wp_bytes) / per_warp);
   if (t_warps < 1) use_t = false;
   int t_grid = 0;
   const int t_smem = wp_bytes + t_warps * per_warp;

@@ -1055,10 +1055,18 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const CC& c, uint8
 // keep), strip g + 1 takes strip g's bottom row only when its first lane continues a pair, and
 // every lane folds its maximum into its pair's entry (atomicMax in shared memory); the lane
 // that completes a pair's last lane emits its scores.
-constexpr int kTQ = 96;      // pairs in a team's ring: W strips x 32 lanes / >= 3 lanes per pair
+// Ring capacity: a warp asking for strip g + W has finished strip g, and every strip before g + 1
+// is finished (its warp moved on), so the unfinished pairs lie in strips g + 1 .. g + W: at most
+// W x 32 / 3 + 1 pairs (>= 3 lanes per pair, n' >= 48).  A ring that small would let the
+// appending warp wait for a pair whose lanes sit in a strip that itself waits for the append
+// (deadlock), so each team gets cap = kTPool / teams >= 32 W / 3 + 2 entries of a per-CTA pool.
+constexpr int kTPool = 112;
 struct TStream {
   int lock, count, next, end;   // next: lanes appended so far
-  int item[kTQ], base[kTQ], nl[kTQ], rem[kTQ], mlo[kTQ], mhi[kTQ];
+  int off, cap;                 // this team's entries: pool[off .. off + cap)
+};
+struct TPool {
+  int item[kTPool], base[kTPool], nl[kTPool], rem[kTPool], mlo[kTPool], mhi[kTPool];
 };
 
 // L = LaneS32: the 32-bit recompute of the flagged sequences (items = positions of
@@ -1067,7 +1075,8 @@ struct TStream {
 template <int C, class L, class CC>
 __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uint8_t* tab,
                                               const int8_t* wp, int W, int team, int wt, int first_item,
-                                              unsigned long long* prog, uint2* rb, TStream* ts) {
+                                              unsigned long long* prog, uint2* rb, TStream* ts, TPool* pool,
+                                              int nteams) {
   constexpr bool S32 = L::kSeqs == 1;
   constexpr int CB = chunk_bytes<C>();
   constexpr int LS = 32 * C;
@@ -1076,6 +1085,8 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
   const int qsteps = (p.qcols + 32 + 3) & ~3;
   const int n_items = S32 ? *p.item_count : p.n_items;
   volatile TStream* vs = ts;
+  volatile TPool* vp = pool;
+  const int cap = kTPool / nteams, off = team * cap;
   // item -> (pair, half): s16x2 items are pairs, s32 items index the flagged-sequence list
   auto pair_of = [&](int item, int* half) {
     if constexpr (S32) {
@@ -1095,10 +1106,10 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
   auto append = [&](int item) {
     int hf;
     const int nl = (p.pair_ncols[pair_of(item, &hf)] + C - 1) / C;   // >= 3 lanes (n' >= 48)
-    const int k = vs->count % kTQ;
-    if (vs->count >= kTQ)   // the entry kTQ pairs back must be finished before it is reused
-      while (vs->rem[k] != 0) __nanosleep(64);
-    vs->item[k] = item; vs->base[k] = vs->next; vs->nl[k] = nl; vs->rem[k] = nl; vs->mlo[k] = 0; vs->mhi[k] = 0;
+    const int k = off + vs->count % cap;
+    if (vs->count >= cap)   // the entry cap pairs back must be finished before it is reused
+      while (vp->rem[k] != 0) __nanosleep(64);
+    vp->item[k] = item; vp->base[k] = vs->next; vp->nl[k] = nl; vp->rem[k] = nl; vp->mlo[k] = 0; vp->mhi[k] = 0;
     __threadfence_block();
     vs->count = vs->count + 1;
     vs->next = vs->next + nl;
@@ -1137,17 +1148,17 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
     int k = -1;
     {
       const int count = vs->count;
-      for (int j = count - 1; j >= 0 && j >= count - kTQ; --j) {
-        const int kk = j % kTQ;
-        if (vs->base[kk] <= gl) { if (gl < vs->base[kk] + vs->nl[kk]) k = kk; break; }
+      for (int j = count - 1; j >= 0 && j >= count - cap; --j) {
+        const int kk = off + j % cap;
+        if (vp->base[kk] <= gl) { if (gl < vp->base[kk] + vp->nl[kk]) k = kk; break; }
       }
     }
     int item = -1, half = 0, pair = 0, ncols = 0, lip = 0;
     if (k >= 0) {
-      item = vs->item[k];
+      item = vp->item[k];
       pair = pair_of(item, &half);
       ncols = p.pair_ncols[pair];
-      lip = gl - vs->base[k];             // lane index within the pair
+      lip = gl - vp->base[k];             // lane index within the pair
     }
     const uint16_t* cp = p.cols + (k >= 0 ? p.pair_off[pair] : 0);
     build_strip_tables<C, L::kSeqs>(p, tab, wp, cp, k >= 0 ? ncols : 0, lip * C, half);
@@ -1161,14 +1172,14 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
                                                        0u, keep);
     if (k >= 0) {
       if constexpr (S32) {
-        atomicMax(&ts->mlo[k], (int)b);
+        atomicMax(&pool->mlo[k], (int)b);
       } else {
-        atomicMax(&ts->mlo[k], (int)(int16_t)(b & 0xffffu));
-        atomicMax(&ts->mhi[k], (int)(int16_t)(b >> 16));
+        atomicMax(&pool->mlo[k], (int)(int16_t)(b & 0xffffu));
+        atomicMax(&pool->mhi[k], (int)(int16_t)(b >> 16));
       }
       __threadfence_block();
-      if (atomicSub(&ts->rem[k], 1) == 1) {   // this pair's last lane
-        const int lo = atomicAdd(&ts->mlo[k], 0), hi = atomicAdd(&ts->mhi[k], 0);
+      if (atomicSub(&pool->rem[k], 1) == 1) {   // this pair's last lane
+        const int lo = atomicAdd(&pool->mlo[k], 0), hi = atomicAdd(&pool->mhi[k], 0);
         emit_item(item, lo, hi);
       }
     }
@@ -1320,8 +1331,9 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   if (team >= nteams) return;
   const int first = (team == 0) ? sparked : -1;
   __shared__ TStream sts[kTmodeThreads / 32];
+  __shared__ TPool spool;
   t_team_stream<C, L>(p, c, tab, wp, W, team, wt, first, sprog64 + team * (W + 1),
-                      rb_cta + (int64_t)team * (W + 1) * p.rb_cols, &sts[team]);
+                      rb_cta + (int64_t)team * (W + 1) * p.rb_cols, &sts[team], &spool, nteams);
 }
 
 template <int C, int NT, bool WIDE, class L>
