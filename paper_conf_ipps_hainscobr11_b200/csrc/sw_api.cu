@@ -13,6 +13,7 @@
 #include <string>
 #include <thread>
 #include <vector>
+#include <unistd.h>
 
 #include "../../include/sw.h"
 #include "sw_internal.h"

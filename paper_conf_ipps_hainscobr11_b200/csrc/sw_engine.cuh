@@ -1110,8 +1110,11 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
     if (vs->count >= cap)   // the entry cap pairs back must be finished before it is reused
       while (vp->rem[k] != 0) __nanosleep(64);
     vp->item[k] = item; vp->base[k] = vs->next; vp->nl[k] = nl; vp->rem[k] = nl; vp->mlo[k] = 0; vp->mhi[k] = 0;
+    // publication order: the entry, then count, then next — a reader that sees next cover its
+    // strip (and fences) sees the count that includes every entry of the strip
     __threadfence_block();
     vs->count = vs->count + 1;
+    __threadfence_block();
     vs->next = vs->next + nl;
   };
   team_bar(team, W);
@@ -1124,10 +1127,16 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
   team_bar(team, W);
   for (int g = wt;; g += W) {
     // strip g needs every pair that covers its lanes (lane 0 appends, the warp follows)
-    int have = 0;
+    int have = 0, count = 0;
     if (lane == 0) {
       for (;;) {
-        if (vs->next >= 32 * g + 32 || vs->end) { have = vs->next > 32 * g; break; }
+        const int nx = vs->next;
+        if (nx >= 32 * g + 32 || vs->end) {
+          __threadfence_block();
+          have = vs->next > 32 * g;
+          count = vs->count;   // read after next (fenced): includes every entry of the strip
+          break;
+        }
         if (atomicCAS(&ts->lock, 0, 1) == 0) {
           while (vs->next < 32 * g + 32 && !vs->end) {
             const int item = p.gang_items + atomicAdd(p.work, 1);
@@ -1142,12 +1151,13 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
       }
     }
     have = __shfl_sync(SWB_FULL, have, 0);
+    count = __shfl_sync(SWB_FULL, count, 0);
     if (!have) break;
+    __threadfence_block();
     // this lane's pair: the newest ring entry starting at or before lane 32g + lane
     const int gl = 32 * g + lane;
     int k = -1;
     {
-      const int count = vs->count;
       for (int j = count - 1; j >= 0 && j >= count - cap; --j) {
         const int kk = off + j % cap;
         if (vp->base[kk] <= gl) { if (gl < vp->base[kk] + vp->nl[kk]) k = kk; break; }
