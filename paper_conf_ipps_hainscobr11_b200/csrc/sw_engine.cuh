@@ -1063,8 +1063,9 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const CC& c, uint8
 constexpr int kTPool = 112;
 struct TStream {
   int lock, count, next, end;   // next: lanes appended so far
-  int off, cap;                 // this team's entries: pool[off .. off + cap)
+  int pend, pend_end;           // queue items taken (kTGrab at a time) but not appended yet
 };
+constexpr int kTGrab = 8;       // queue items per global atomic
 struct TPool {
   int item[kTPool], base[kTPool], nl[kTPool], rem[kTPool], mlo[kTPool], mhi[kTPool];
 };
@@ -1102,10 +1103,13 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
     if constexpr (S32) emit_t32(p, lo, p.item_list[item]);
     else emit_t(p, ((uint32_t)lo & 0xffffu) | ((uint32_t)hi << 16), item);
   };
-  // append one pair to the ring (lane 0 of the warp holding the lock)
+  // append one pair to the ring (lane 0 of the warp holding the lock).  A pair of a strip or more
+  // starts a new strip (the lanes skipped are pad lanes): its first strip then depends on no
+  // other strip, as in the one-pair-per-strip layout; shorter pairs are packed back to back.
   auto append = [&](int item) {
     int hf;
     const int nl = (p.pair_ncols[pair_of(item, &hf)] + C - 1) / C;   // >= 3 lanes (n' >= 48)
+    if (nl >= 32 && (vs->next & 31)) vs->next = (vs->next + 31) & ~31;
     const int k = off + vs->count % cap;
     if (vs->count >= cap)   // the entry cap pairs back must be finished before it is reused
       while (vp->rem[k] != 0) __nanosleep(64);
@@ -1117,10 +1121,20 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
     __threadfence_block();
     vs->next = vs->next + nl;
   };
+  // the next queue item (kTGrab items per global atomic; -1 at the end)
+  auto take = [&]() -> int {
+    if (vs->pend == vs->pend_end) {
+      const int b0 = atomicAdd(p.work, kTGrab);
+      vs->pend = b0; vs->pend_end = b0 + kTGrab;
+    }
+    const int item = p.gang_items + vs->pend;
+    vs->pend = vs->pend + 1;
+    return item < n_items ? item : -1;
+  };
   team_bar(team, W);
   if (wt == 0 && lane == 0) {
     for (int i = 0; i <= W; ++i) prog[i] = 0u;
-    ts->lock = 0; ts->count = 0; ts->next = 0; ts->end = 0;
+    ts->lock = 0; ts->count = 0; ts->next = 0; ts->end = 0; ts->pend = 0; ts->pend_end = 0;
     if (first_item >= 0) append(first_item);
     __threadfence_block();
   }
@@ -1138,9 +1152,17 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
           break;
         }
         if (atomicCAS(&ts->lock, 0, 1) == 0) {
-          while (vs->next < 32 * g + 32 && !vs->end) {
-            const int item = p.gang_items + atomicAdd(p.work, 1);
-            if (item >= n_items) { vs->end = 1; break; }
+          while (vs->next < 32 * g + 32 && !vs->end) {   // this strip's pairs (may wait for the ring)
+            const int item = take();
+            if (item < 0) { vs->end = 1; break; }
+            append(item);
+          }
+          // look ahead for the team's next strips while ring entries are free (never waits:
+          // the oldest entry may lie in this warp's own, not yet processed, strip)
+          while (vs->next < 32 * (g + W) + 32 && !vs->end &&
+                 (vs->count < cap || vp->rem[off + vs->count % cap] == 0)) {
+            const int item = take();
+            if (item < 0) { vs->end = 1; break; }
             append(item);
           }
           __threadfence_block();
