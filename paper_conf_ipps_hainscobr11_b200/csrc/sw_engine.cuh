@@ -1121,11 +1121,18 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
     __threadfence_block();
     vs->next = vs->next + nl;
   };
-  // the next queue item (kTGrab items per global atomic; -1 at the end)
+  // the next queue item (-1 at the end).  Pairs shorter than a strip are taken kTGrab per
+  // global atomic (one atomic round trip per pair was on every strip's critical path); longer
+  // ones one at a time, so that the teams stay balanced at the end of the queue (items come
+  // longest first, so the length of the item at the counter tells which case applies)
   auto take = [&]() -> int {
     if (vs->pend == vs->pend_end) {
-      const int b0 = atomicAdd(p.work, kTGrab);
-      vs->pend = b0; vs->pend_end = b0 + kTGrab;
+      const int cur = *reinterpret_cast<volatile int*>(p.work) + p.gang_items;
+      int hf = 0;
+      const bool short_pairs = cur < n_items && p.pair_ncols[pair_of(cur, &hf)] < 32 * C;
+      const int grab = short_pairs ? kTGrab : 1;
+      const int b0 = atomicAdd(p.work, grab);
+      vs->pend = b0; vs->pend_end = b0 + grab;
     }
     const int item = p.gang_items + vs->pend;
     vs->pend = vs->pend + 1;
@@ -1154,7 +1161,7 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
         if (atomicCAS(&ts->lock, 0, 1) == 0) {
           while (vs->next < 32 * g + 32 && !vs->end) {   // this strip's pairs (may wait for the ring)
             const int item = take();
-            if (item < 0) { vs->end = 1; break; }
+            if (item < 0) { __threadfence_block(); vs->end = 1; break; }   // end after the last next
             append(item);
           }
           // look ahead for the team's next strips while ring entries are free (never waits:
@@ -1162,7 +1169,7 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
           while (vs->next < 32 * (g + W) + 32 && !vs->end &&
                  (vs->count < cap || vp->rem[off + vs->count % cap] == 0)) {
             const int item = take();
-            if (item < 0) { vs->end = 1; break; }
+            if (item < 0) { __threadfence_block(); vs->end = 1; break; }   // end after the last next
             append(item);
           }
           __threadfence_block();
