@@ -831,6 +831,8 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     t.rb = s.d_rb_t;
     t.rb_cols = qcols + kPadCols + 1;
     t.hi_mul = 1u << 24;
+    t.pack_flags = 7;
+    if (const char* f = getenv("SW_T_PACK_FLAGS")) t.pack_flags = atoi(f);
     if (t.gang_items > 0) SW_CUDA(h, cudaStreamWaitEvent(tst, h->gang_ev, 0));
     SW_CUDA(h, cudaEventRecord(ev[3], tst));
     SW_CUDA(h, launch_tmode(t, t_grid, t_smem, tst));

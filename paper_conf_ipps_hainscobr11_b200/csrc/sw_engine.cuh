@@ -1109,11 +1109,13 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
   auto append = [&](int item) {
     int hf;
     const int nl = (p.pair_ncols[pair_of(item, &hf)] + C - 1) / C;   // >= 3 lanes (n' >= 48)
-    if (nl >= 32 && (vs->next & 31)) vs->next = (vs->next + 31) & ~31;
+    if ((p.pack_flags & 4) && nl >= 32 && (vs->next & 31)) vs->next = (vs->next + 31) & ~31;
     const int k = off + vs->count % cap;
     if (vs->count >= cap)   // the entry cap pairs back must be finished before it is reused
       while (vp->rem[k] != 0) __nanosleep(64);
-    vp->item[k] = item; vp->base[k] = vs->next; vp->nl[k] = nl; vp->rem[k] = nl; vp->mlo[k] = 0; vp->mhi[k] = 0;
+    // rem = lanes + 1: the lane that completes the pair emits first and then releases the entry
+    // (the appender recycles an entry only at rem == 0, after its maxima were read)
+    vp->item[k] = item; vp->base[k] = vs->next; vp->nl[k] = nl; vp->rem[k] = nl + 1; vp->mlo[k] = 0; vp->mhi[k] = 0;
     // publication order: the entry, then count, then next — a reader that sees next cover its
     // strip (and fences) sees the count that includes every entry of the strip
     __threadfence_block();
@@ -1130,7 +1132,7 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
       const int cur = *reinterpret_cast<volatile int*>(p.work) + p.gang_items;
       int hf = 0;
       const bool short_pairs = cur < n_items && p.pair_ncols[pair_of(cur, &hf)] < 32 * C;
-      const int grab = short_pairs ? kTGrab : 1;
+      const int grab = (short_pairs && (p.pack_flags & 1)) ? kTGrab : 1;
       const int b0 = atomicAdd(p.work, grab);
       vs->pend = b0; vs->pend_end = b0 + grab;
     }
@@ -1166,7 +1168,7 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
           }
           // look ahead for the team's next strips while ring entries are free (never waits:
           // the oldest entry may lie in this warp's own, not yet processed, strip)
-          while (vs->next < 32 * (g + W) + 32 && !vs->end &&
+          while ((p.pack_flags & 2) && vs->next < 32 * (g + W) + 32 && !vs->end &&
                  (vs->count < cap || vp->rem[off + vs->count % cap] == 0)) {
             const int item = take();
             if (item < 0) { __threadfence_block(); vs->end = 1; break; }   // end after the last next
@@ -1217,9 +1219,11 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
         atomicMax(&pool->mhi[k], (int)(int16_t)(b >> 16));
       }
       __threadfence_block();
-      if (atomicSub(&pool->rem[k], 1) == 1) {   // this pair's last lane
+      if (atomicSub(&pool->rem[k], 1) == 2) {   // this pair's last lane
         const int lo = atomicAdd(&pool->mlo[k], 0), hi = atomicAdd(&pool->mhi[k], 0);
         emit_item(item, lo, hi);
+        __threadfence_block();
+        atomicSub(&pool->rem[k], 1);             // release the entry
       }
     }
     __syncwarp();
