@@ -97,20 +97,20 @@ def test_async_device_pointer_and_stream():
         assert km["search_ms"] > 0
 
 
-def test_unsupported_parameter_ranges():
-    with pytest.raises(swp.SWError) as e:
-        swp.sw_create(gen.make_query(10), BLOSUM62, 120, 1)     # 120 + 11 > 127: int8 profile range
-    assert e.value.status == swp.SW_E_UNSUPPORTED
-    # a query whose profile cannot be staged in shared memory is refused, never computed on the CPU
-    h = swp.sw_create(gen.make_query(20000), BLOSUM62, 10, 2)
-    try:
-        db = _db(20)
-        swp.sw_load_db(h, db.residues, db.offsets)
-        with pytest.raises(swp.SWError) as e:
-            swp.sw_search(h, db.num_seqs, 3072)
-        assert e.value.status == swp.SW_E_UNSUPPORTED
-    finally:
-        swp.sw_destroy(h)
+def test_formerly_unsupported_parameter_ranges_now_search():
+    """Round 1 refused rho + max(w) > 127 (the int8 profile range) and queries whose profile does
+    not fit shared memory; both now run (WIDE kernels, long-query mode) with exact scores —
+    and never on the CPU (tests/test_wide_params_gpu.py, tests/test_long_query_gpu.py)."""
+    import oracle
+    db = _db(20)
+    for q, rho in ((gen.make_query(10), 120), (gen.make_query(20000), 10)):
+        h = swp.sw_create(q, BLOSUM62, rho, 1)
+        try:
+            swp.sw_load_db(h, db.residues, db.offsets)
+            got = swp.sw_search(h, db.num_seqs, 3072)
+        finally:
+            swp.sw_destroy(h)
+        assert np.array_equal(got, oracle.scores(q, BLOSUM62, rho, 1, db.residues, db.offsets))
 
 
 def test_version_and_null_destroy():
