@@ -831,8 +831,14 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     t.rb = s.d_rb_t;
     t.rb_cols = qcols + kPadCols + 1;
     t.hi_mul = 1u << 24;
-    t.pack_flags = 7;
-    if (const char* f = getenv("SW_T_PACK_FLAGS")) t.pack_flags = atoi(f);
+    // team-stream layout: packed lanes when the long pairs average under two strips (their
+    // one-pair-per-strip padding is large: C2 at T = 512, 3604 vs 2961 GCUPS), one pair per
+    // strip otherwise (C2 at T = 3072: 1.24 vs 0.97 ms; profiles/r02_tmode_packed.txt)
+    {
+      const double mean_cols = n_long ? (double)sp.long_cols / n_long : 0.0;
+      t.packed = mean_cols < 2.0 * 32 * kTmodeC;
+      if (const char* f = getenv("SW_T_PACKED")) t.packed = atoi(f) != 0;
+    }
     if (t.gang_items > 0) SW_CUDA(h, cudaStreamWaitEvent(tst, h->gang_ev, 0));
     SW_CUDA(h, cudaEventRecord(ev[3], tst));
     SW_CUDA(h, launch_tmode(t, t_grid, t_smem, tst));

@@ -1047,6 +1047,124 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const CC& c, uint8
 // (slot g mod (W + 1), tag = g): strip g + 1 consumes strip g's bottom row only inside a pair.
 // Each pair's maximum is combined with atomicMax in the team's shared ring of pairs; the
 // warp finishing its last strip emits the scores.
+// Per-pair team stream (used when the long pairs are a strip or more on average): every pair
+// starts a new strip, strips of one pair are chained, a new pair's first strip depends on no
+// other strip.  (The packed stream below is used for long sets of mostly short pairs.)
+constexpr int kTQ = 16;      // pairs in a team's ring (a team spans at most ~W + 1 of them)
+struct TStreamP {
+  int lock, count, next, end;
+  int item[kTQ], base[kTQ], S[kTQ], rem[kTQ], mlo[kTQ], mhi[kTQ];
+};
+
+// L = LaneS32: the 32-bit recompute of the flagged sequences (items = positions of
+// p.item_list, one sequence each; long-query mode, where the k_search recompute's query profile
+// does not fit shared memory).  Progress tags are 64-bit (running strip index << 32 | columns).
+template <int C, class L, class CC>
+__device__ __forceinline__ void t_team_stream_pairs(const TParams& p, const CC& c, uint8_t* tab,
+                                                    const int8_t* wp, int W, int team, int wt, int first_item,
+                                                    unsigned long long* prog, uint2* rb, TStreamP* ts) {
+  constexpr bool S32 = L::kSeqs == 1;
+  constexpr int CB = chunk_bytes<C>();
+  constexpr int LS = 32 * C;
+  const int lane = threadIdx.x & 31;
+  const int A1 = p.A_used + 1;
+  const int qsteps = (p.qcols + 32 + 3) & ~3;
+  const int n_items = S32 ? *p.item_count : p.n_items;
+  volatile TStreamP* vs = ts;
+  // item -> (pair, half): s16x2 items are pairs, s32 items index the flagged-sequence list
+  auto pair_of = [&](int item, int* half) {
+    if constexpr (S32) {
+      const int sq = p.item_list[item];
+      *half = sq & 1;
+      return sq >> 1;
+    } else {
+      *half = 0;
+      return item;
+    }
+  };
+  auto emit_item = [&](int item, int lo, int hi) {
+    if constexpr (S32) emit_t32(p, lo, p.item_list[item]);
+    else emit_t(p, ((uint32_t)lo & 0xffffu) | ((uint32_t)hi << 16), item);
+  };
+  // append one pair to the ring (lane 0 of the warp holding the lock); empty pairs score 0
+  auto append = [&](int item) {
+    int hf;
+    const int S = (p.pair_ncols[pair_of(item, &hf)] + LS - 1) / LS;
+    if (S == 0) { emit_item(item, 0, 0); return; }
+    const int k = vs->count % kTQ;
+    if (vs->count >= kTQ)   // the entry kTQ pairs back must be finished before it is reused
+      while (vs->rem[k] != 0) __nanosleep(64);
+    vs->item[k] = item; vs->base[k] = vs->next; vs->S[k] = S; vs->rem[k] = S; vs->mlo[k] = 0; vs->mhi[k] = 0;
+    __threadfence_block();
+    vs->count = vs->count + 1;
+    vs->next = vs->next + S;
+  };
+  team_bar(team, W);
+  if (wt == 0 && lane == 0) {
+    for (int i = 0; i <= W; ++i) prog[i] = 0u;
+    ts->lock = 0; ts->count = 0; ts->next = 0; ts->end = 0;
+    if (first_item >= 0) append(first_item);
+    __threadfence_block();
+  }
+  team_bar(team, W);
+  for (int g = wt;; g += W) {
+    // the ring entry of strip g (lane 0 decides, the warp follows)
+    int k = -1;
+    if (lane == 0) {
+      for (;;) {
+        const int next = vs->next, count = vs->count;
+        if (g < next) {
+          for (int j = count - 1; j >= 0 && j >= count - kTQ; --j) {
+            const int kk = j % kTQ;
+            if (vs->base[kk] <= g) { k = kk; break; }
+          }
+          break;
+        }
+        if (vs->end) break;
+        if (atomicCAS(&ts->lock, 0, 1) == 0) {
+          while (vs->next <= g && !vs->end) {
+            const int item = p.gang_items + atomicAdd(p.work, 1);
+            if (item >= n_items) { vs->end = 1; break; }
+            append(item);
+          }
+          __threadfence_block();
+          atomicExch(&ts->lock, 0);
+        } else {
+          __nanosleep(64);
+        }
+      }
+    }
+    k = __shfl_sync(SWB_FULL, k, 0);
+    if (k < 0) break;
+    const int item = vs->item[k], P = g - vs->base[k], S = vs->S[k];
+    int half;
+    const int pair = pair_of(item, &half);
+    const int ncols = p.pair_ncols[pair];
+    const uint16_t* cp = p.cols + p.pair_off[pair];
+    build_strip_tables<C, L::kSeqs>(p, tab, wp, cp, ncols, P * LS + lane * C, half);
+    const int si = (g + W) % (W + 1), so = g % (W + 1);
+    uint32_t b = run_pass<L, 32, C, true, 4, false, 32>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps,
+                                                       P, S, rb + (int64_t)si * p.rb_cols + 1,
+                                                       rb + (int64_t)so * p.rb_cols + 1, prog + si, prog + so, 0u, g);
+#pragma unroll
+    for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
+    if (lane == 0) {
+      if constexpr (S32) {
+        atomicMax(&ts->mlo[k], (int)b);
+      } else {
+        atomicMax(&ts->mlo[k], (int)(int16_t)(b & 0xffffu));
+        atomicMax(&ts->mhi[k], (int)(int16_t)(b >> 16));
+      }
+      __threadfence_block();
+      if (atomicSub(&ts->rem[k], 1) == 1) {   // this pair's last strip
+        const int lo = atomicAdd(&ts->mlo[k], 0), hi = atomicAdd(&ts->mhi[k], 0);
+        emit_item(item, lo, hi);
+      }
+    }
+    __syncwarp();
+  }
+}
+
 // PACKED: the team's pairs are laid out back to back in LANES of C database positions (a pair
 // of n' columns takes ceil(n' / C) lanes) and strip g is the team's lanes [32g, 32g + 32): a
 // strip holds the tail of one pair and the heads of the next ones, so short pairs no longer
@@ -1103,13 +1221,10 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
     if constexpr (S32) emit_t32(p, lo, p.item_list[item]);
     else emit_t(p, ((uint32_t)lo & 0xffffu) | ((uint32_t)hi << 16), item);
   };
-  // append one pair to the ring (lane 0 of the warp holding the lock).  A pair of a strip or more
-  // starts a new strip (the lanes skipped are pad lanes): its first strip then depends on no
-  // other strip, as in the one-pair-per-strip layout; shorter pairs are packed back to back.
+  // append one pair to the ring (lane 0 of the warp holding the lock)
   auto append = [&](int item) {
     int hf;
     const int nl = (p.pair_ncols[pair_of(item, &hf)] + C - 1) / C;   // >= 3 lanes (n' >= 48)
-    if ((p.pack_flags & 4) && nl >= 32 && (vs->next & 31)) vs->next = (vs->next + 31) & ~31;
     const int k = off + vs->count % cap;
     if (vs->count >= cap)   // the entry cap pairs back must be finished before it is reused
       while (vp->rem[k] != 0) __nanosleep(64);
@@ -1132,7 +1247,7 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
       const int cur = *reinterpret_cast<volatile int*>(p.work) + p.gang_items;
       int hf = 0;
       const bool short_pairs = cur < n_items && p.pair_ncols[pair_of(cur, &hf)] < 32 * C;
-      const int grab = (short_pairs && (p.pack_flags & 1)) ? kTGrab : 1;
+      const int grab = short_pairs ? kTGrab : 1;
       const int b0 = atomicAdd(p.work, grab);
       vs->pend = b0; vs->pend_end = b0 + grab;
     }
@@ -1162,14 +1277,6 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
         }
         if (atomicCAS(&ts->lock, 0, 1) == 0) {
           while (vs->next < 32 * g + 32 && !vs->end) {   // this strip's pairs (may wait for the ring)
-            const int item = take();
-            if (item < 0) { __threadfence_block(); vs->end = 1; break; }   // end after the last next
-            append(item);
-          }
-          // look ahead for the team's next strips while ring entries are free (never waits:
-          // the oldest entry may lie in this warp's own, not yet processed, strip)
-          while ((p.pack_flags & 2) && vs->next < 32 * (g + W) + 32 && !vs->end &&
-                 (vs->count < cap || vp->rem[off + vs->count % cap] == 0)) {
             const int item = take();
             if (item < 0) { __threadfence_block(); vs->end = 1; break; }   // end after the last next
             append(item);
@@ -1373,10 +1480,16 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   const int team = (warp - wbase) / W, wt = (warp - wbase) % W;
   if (team >= nteams) return;
   const int first = (team == 0) ? sparked : -1;
-  __shared__ TStream sts[kTmodeThreads / 32];
-  __shared__ TPool spool;
-  t_team_stream<C, L>(p, c, tab, wp, W, team, wt, first, sprog64 + team * (W + 1),
-                      rb_cta + (int64_t)team * (W + 1) * p.rb_cols, &sts[team], &spool, nteams);
+  if (p.packed) {
+    __shared__ TStream sts[kTmodeThreads / 32];
+    __shared__ TPool spool;
+    t_team_stream<C, L>(p, c, tab, wp, W, team, wt, first, sprog64 + team * (W + 1),
+                        rb_cta + (int64_t)team * (W + 1) * p.rb_cols, &sts[team], &spool, nteams);
+  } else {
+    __shared__ TStreamP stsp[kTmodeThreads / 32];
+    t_team_stream_pairs<C, L>(p, c, tab, wp, W, team, wt, first, sprog64 + team * (W + 1),
+                              rb_cta + (int64_t)team * (W + 1) * p.rb_cols, &stsp[team]);
+  }
 }
 
 template <int C, int NT, bool WIDE, class L>

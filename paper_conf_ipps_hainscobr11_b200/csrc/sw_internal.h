@@ -138,7 +138,7 @@ struct TParams {
   int gang_items, gang_ctas, gang_warps;
   int gang_share;            // 1: the gang CTAs' other warps run the team stream meanwhile
   int gang_chain2;           // 1: the gang warps use the two-op vertical chain (cell_rows CHAIN2)
-  int pack_flags;            // team stream: 1 batch queue takes, 2 look-ahead appends, 4 strip-aligned long pairs
+  int packed;                // team stream layout: 1 packed lanes (mostly short pairs), 0 one pair per strip
   uint32_t gang_epoch;       // tag epoch of this launch's hand-off words (20 bits, != the last launch's)
   unsigned long long* dbg_times;   // probe (SW_DEBUG_GANG_TIMES): gang item 0's strip start / end (ns)
   int32_t* gang_ctr;         // slot counter
