@@ -34,6 +34,8 @@ if len(sys.argv) > 6 and sys.argv[6]:
 off = np.concatenate([[0], np.cumsum(L[idx])]).astype(np.int64)
 res = np.concatenate([db.residues[db.offsets[i]:db.offsets[i + 1]] for i in idx])
 q = gen.make_query(m)
+if os.environ.get("SW_LIB"):          # A/B against another build of the library
+    swp.load_library(os.environ["SW_LIB"])
 with swp.SmithWaterman(q, BLOSUM62, 10, 2) as sw:
     sw.load_db(res, off)
     for _ in range(reps):
