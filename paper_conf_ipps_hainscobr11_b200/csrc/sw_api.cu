@@ -588,9 +588,14 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
   if (t_warps < 1) use_t = false;
   int t_grid = 0;
   const int t_smem = wp_bytes + t_warps * per_warp;
+  // team-stream layout (a compile-time variant of k_search_t): packed lanes when the long pairs
+  // average under two strips (their one-pair-per-strip padding is large: C2 at T = 512, 3586 vs
+  // 2966 GCUPS), one pair per strip otherwise (profiles/r02_tmode_packed.txt)
+  bool t_packed = n_long > 0 && (double)sp.long_cols / n_long < 2.0 * 32 * kTmodeC;
+  if (const char* f = getenv("SW_T_PACKED")) t_packed = atoi(f) != 0;
   if (use_t) {
     int bps = 0;
-    cudaError_t e = configure_tmode_kernel(t_smem, &bps, h->wide);
+    cudaError_t e = configure_tmode_kernel(t_smem, &bps, h->wide, false, t_packed);
     if (e != cudaSuccess) return cuda_fail(h, e, "configure long-sequence kernel");
     t_grid = std::max(1, bps) * h->num_sms;
     rc = grow(h, &s.d_qpair, &s.qpair_cap, (size_t)(qcols + kPadCols) * sizeof(uint16_t), "alloc query stream",
@@ -831,14 +836,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     t.rb = s.d_rb_t;
     t.rb_cols = qcols + kPadCols + 1;
     t.hi_mul = 1u << 24;
-    // team-stream layout: packed lanes when the long pairs average under two strips (their
-    // one-pair-per-strip padding is large: C2 at T = 512, 3604 vs 2961 GCUPS), one pair per
-    // strip otherwise (C2 at T = 3072: 1.24 vs 0.97 ms; profiles/r02_tmode_packed.txt)
-    {
-      const double mean_cols = n_long ? (double)sp.long_cols / n_long : 0.0;
-      t.packed = mean_cols < 2.0 * 32 * kTmodeC;
-      if (const char* f = getenv("SW_T_PACKED")) t.packed = atoi(f) != 0;
-    }
+    t.packed = t_packed;
     if (t.gang_items > 0) SW_CUDA(h, cudaStreamWaitEvent(tst, h->gang_ev, 0));
     SW_CUDA(h, cudaEventRecord(ev[3], tst));
     SW_CUDA(h, launch_tmode(t, t_grid, t_smem, tst));
@@ -871,7 +869,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
       while (t.warps % r.team_warps) --r.team_warps;
       const int smem32 = wp_bytes + t.warps * per_warp / 2;
       int bps = 0;
-      cudaError_t e = configure_tmode_kernel(smem32, &bps, h->wide, true);
+      cudaError_t e = configure_tmode_kernel(smem32, &bps, h->wide, true, r.packed);
       if (e != cudaSuccess) return cuda_fail(h, e, "configure long-sequence recompute kernel");
       SW_CUDA(h, launch_tmode(r, std::min(t_grid, std::max(1, bps) * h->num_sms), smem32, st, true));
       SW_CUDA(h, cudaEventRecord(ev[2], st));

@@ -37,6 +37,9 @@
 namespace swb {
 
 #define SWB_FULL 0xffffffffu
+// packed T-mode team stream's progress tags (strip << 33 | columns); the distinct shift also
+// enables run_pass's per-lane keep mask (sw_engine.cuh t_team_stream)
+constexpr int kPackedTagShift = 33;
 
 // PRMT with a compile-time selector.  Inline PTX because __byte_perm keeps only 3 bits per
 // selector nibble, while the 4th bit (sign replication of the selected byte) is what turns
@@ -467,7 +470,7 @@ __device__ __forceinline__ uint32_t run_pass(const CC& c, const uint8_t* prow, i
       if (gl == 0) x_res = rr[K];
     } else {
       if (gl == 0) { x_hr = rh[K]; x_f = rf[K]; x_res = rr[K]; }
-      if constexpr (TAG_SHIFT == 32) { x_hr *= keep; x_f *= keep; }   // (IMAD) packed team stream
+      if constexpr (TAG_SHIFT == kPackedTagShift) { x_hr *= keep; x_f *= keep; }   // (IMAD) packed stream
     }
     // query-profile words for the two letters of the NEXT column (look-ahead u)
     uint32_t wlo[(R + 3) / 4], whi[(R + 3) / 4];
@@ -1314,8 +1317,8 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
     const int cont = __shfl_sync(SWB_FULL, k >= 0 && lip > 0 ? 1 : 0, 0);
     const uint32_t keep = (lane > 0 && k >= 0 && lip == 0) ? 0u : 1u;
     const int si = (g + W) % (W + 1), so = g % (W + 1);
-    uint32_t b = run_pass<L, 32, C, true, 4, false, 32>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols, 0, qsteps,
-                                                       cont, 3, rb + (int64_t)si * p.rb_cols + 1,
+    uint32_t b = run_pass<L, 32, C, true, 4, false, kPackedTagShift>(c, tab + lane * CB, LS, A1 * LS, p.qpair, p.qcols,
+                                                                    0, qsteps, cont, 3, rb + (int64_t)si * p.rb_cols + 1,
                                                        rb + (int64_t)so * p.rb_cols + 1, prog + si, prog + so, 0u, g,
                                                        0u, keep);
     if (k >= 0) {
@@ -1404,7 +1407,9 @@ __device__ __forceinline__ void t_gang_item(const TParams& p, const CC& c, uint8
   }
 }
 
-template <int C, int NT, bool WIDE = false, class L = LaneS16x2>
+// PACKED: the team stream's layout (compile-time, one stream per kernel: both in one kernel
+// measured 15-30 % slower for either, code size)
+template <int C, int NT, bool WIDE = false, class L = LaneS16x2, bool PACKED = false>
 __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   constexpr int kWarps = NT / 32;
   constexpr int LS = 32 * C;
@@ -1480,7 +1485,7 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   const int team = (warp - wbase) / W, wt = (warp - wbase) % W;
   if (team >= nteams) return;
   const int first = (team == 0) ? sparked : -1;
-  if (p.packed) {
+  if constexpr (PACKED) {
     __shared__ TStream sts[kTmodeThreads / 32];
     __shared__ TPool spool;
     t_team_stream<C, L>(p, c, tab, wp, W, team, wt, first, sprog64 + team * (W + 1),
@@ -1492,18 +1497,19 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   }
 }
 
-template <int C, int NT, bool WIDE, class L>
+template <int C, int NT, bool WIDE, class L, bool PACKED>
 cudaError_t launch_search_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st) {
-  k_search_t<C, NT, WIDE, L><<<grid, NT, smem_bytes, st>>>(p);
+  k_search_t<C, NT, WIDE, L, PACKED><<<grid, NT, smem_bytes, st>>>(p);
   return cudaGetLastError();
 }
 
-template <int C, int NT, bool WIDE, class L>
+template <int C, int NT, bool WIDE, class L, bool PACKED>
 cudaError_t configure_tmode(int smem_bytes, int* blocks_per_sm) {
-  cudaError_t e =
-      cudaFuncSetAttribute(k_search_t<C, NT, WIDE, L>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+  cudaError_t e = cudaFuncSetAttribute(k_search_t<C, NT, WIDE, L, PACKED>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search_t<C, NT, WIDE, L>, NT, smem_bytes);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search_t<C, NT, WIDE, L, PACKED>, NT,
+                                                       smem_bytes);
 }
 
 template <class L, int G, int Rs, int Rl, int NT, bool WIDE>

@@ -149,7 +149,8 @@ struct TParams {
 };
 
 cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st, bool s32 = false);
-cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm, bool wide, bool s32 = false);
+cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm, bool wide, bool s32 = false,
+                                   bool packed = false);
 cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, uint32_t qmask, cudaStream_t st);
 
 // Traceback of one pair (sw_traceback.cu): dir = m*n bytes, scratch = 7*m ints, result = 6 ints.

@@ -21,23 +21,29 @@ cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, uint32_t
   return cudaGetLastError();
 }
 
-// s32 = true: the 32-bit recompute of the flagged sequences (p.item_list / p.item_count)
-cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st, bool s32) {
-  if (s32) {
-    if (p.delta > 0) return launch_search_tmode<kTmodeC, kTmodeThreads, true, LaneS32>(p, grid, smem_bytes, st);
-    return launch_search_tmode<kTmodeC, kTmodeThreads, false, LaneS32>(p, grid, smem_bytes, st);
-  }
-  if (p.delta > 0) return launch_search_tmode<kTmodeC, kTmodeThreads, true, LaneS16x2>(p, grid, smem_bytes, st);
-  return launch_search_tmode<kTmodeC, kTmodeThreads, false, LaneS16x2>(p, grid, smem_bytes, st);
+// s32 = true: the 32-bit recompute of the flagged sequences (p.item_list / p.item_count);
+// p.packed selects the team stream's layout, p.delta > 0 the WIDE instantiation
+template <bool WIDE, class L>
+static cudaError_t launch_t(const TParams& p, int grid, int smem_bytes, cudaStream_t st) {
+  if (p.packed) return launch_search_tmode<kTmodeC, kTmodeThreads, WIDE, L, true>(p, grid, smem_bytes, st);
+  return launch_search_tmode<kTmodeC, kTmodeThreads, WIDE, L, false>(p, grid, smem_bytes, st);
+}
+template <bool WIDE, class L>
+static cudaError_t configure_t2(int smem_bytes, int* blocks_per_sm, bool packed) {
+  if (packed) return configure_tmode<kTmodeC, kTmodeThreads, WIDE, L, true>(smem_bytes, blocks_per_sm);
+  return configure_tmode<kTmodeC, kTmodeThreads, WIDE, L, false>(smem_bytes, blocks_per_sm);
 }
 
-cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm, bool wide, bool s32) {
-  if (s32) {
-    if (wide) return configure_tmode<kTmodeC, kTmodeThreads, true, LaneS32>(smem_bytes, blocks_per_sm);
-    return configure_tmode<kTmodeC, kTmodeThreads, false, LaneS32>(smem_bytes, blocks_per_sm);
-  }
-  if (wide) return configure_tmode<kTmodeC, kTmodeThreads, true, LaneS16x2>(smem_bytes, blocks_per_sm);
-  return configure_tmode<kTmodeC, kTmodeThreads, false, LaneS16x2>(smem_bytes, blocks_per_sm);
+cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st, bool s32) {
+  if (s32) return p.delta > 0 ? launch_t<true, LaneS32>(p, grid, smem_bytes, st) : launch_t<false, LaneS32>(p, grid, smem_bytes, st);
+  return p.delta > 0 ? launch_t<true, LaneS16x2>(p, grid, smem_bytes, st) : launch_t<false, LaneS16x2>(p, grid, smem_bytes, st);
+}
+
+cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm, bool wide, bool s32, bool packed) {
+  if (s32) return wide ? configure_t2<true, LaneS32>(smem_bytes, blocks_per_sm, packed)
+                       : configure_t2<false, LaneS32>(smem_bytes, blocks_per_sm, packed);
+  return wide ? configure_t2<true, LaneS16x2>(smem_bytes, blocks_per_sm, packed)
+              : configure_t2<false, LaneS16x2>(smem_bytes, blocks_per_sm, packed);
 }
 
 }  // namespace swb
