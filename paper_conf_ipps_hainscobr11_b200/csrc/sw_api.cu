@@ -589,9 +589,12 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
   int t_grid = 0;
   const int t_smem = wp_bytes + t_warps * per_warp;
   // team-stream layout (a compile-time variant of k_search_t): packed lanes when the long pairs
-  // average under two strips (their one-pair-per-strip padding is large: C2 at T = 512, 3586 vs
-  // 2966 GCUPS), one pair per strip otherwise (profiles/r02_tmode_packed.txt)
-  bool t_packed = n_long > 0 && (double)sp.long_cols / n_long < 2.0 * 32 * kTmodeC;
+  // average one to three strips (their one-pair-per-strip padding is large and they hand off
+  // between strips anyway: C2 at T = 512, 3558 vs 2962 GCUPS); one pair per strip otherwise —
+  // longer pairs (T = 1172: 3553 vs 3413; T = 3072: 0.96 vs 1.23 ms) and sub-strip pairs, whose
+  // strips then need no hand-off at all (T = 0: 2147 vs 1966) (profiles/r02_tmode_packed.txt)
+  const double t_mean_cols = n_long > 0 ? (double)sp.long_cols / n_long : 0.0;
+  bool t_packed = t_mean_cols >= 32 * kTmodeC && t_mean_cols < 3.0 * 32 * kTmodeC;
   if (const char* f = getenv("SW_T_PACKED")) t_packed = atoi(f) != 0;
   if (use_t) {
     int bps = 0;
