@@ -675,6 +675,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
       SW_CUDA(h, cudaStreamWaitEvent(s.aux, s.fork, 0));
     }
     TParams t{};
+    std::vector<int32_t> h_gang_base;   // per-gang CTA slot offsets (uploaded with the gang scratch)
     t.matrix = h->d_matrix;
     t.A = h->A;
     t.rho = h->rho16;
@@ -763,6 +764,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
         t_thr /= nw;
         const bool hidden = (double)sp.short_cols > 0.5 * (double)sp.long_cols;
         int K = 0, items = 0;
+        std::vector<int> Ks;   // CTAs of each gang (the longest pairs need more than the others)
         if (!hidden) {
           // a gang of GW warps: each warp runs ceil(S / GW) strips back to back after a ramp of
           // (GW - 1) lags, unless the wavefront (S - 1) lag + qsteps is longer (measured per
@@ -781,26 +783,38 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
             const double goal = std::max(1.15 * t_thr, 1.03 * best_g);
             int k = 2;
             while (k < kMaxGangCtas && gang_time(k * WG, S) > goal) ++k;
+            // the 4-bit hand-off tags (run_pass GPU_FLAGS) repeat every 15 strips: a slot is
+            // reused every GW + 1 strips, which must not be a multiple of 15
+            while (k > 2 && (k * WG + 1) % 15 == 0) --k;
+            if ((k * WG + 1) % 15 == 0) break;
+            Ks.push_back(k);
             K = std::max(K, k);
             ++items;
           }
-          while (items > 0 && items * K > t_grid / 2) --items;
+          int total = 0;
+          for (int i = 0; i < items; ++i) total += Ks[i];
+          while (items > 0 && total > t_grid / 2) total -= Ks[--items];
+          Ks.resize(items);
         }
-        if (const char* f = getenv("SW_T_GANG")) {   // tests: "K" or "K:items"
+        if (const char* f = getenv("SW_T_GANG")) {   // tests: "K" or "K:items" (one size for all)
           K = atoi(f);
+          while (K >= 2 && (K * WG + 1) % 15 == 0) --K;
           const char* comma = strchr(f, ':');
           items = comma ? atoi(comma + 1) : n_long;
           items = std::min(items, std::min(n_long, t_grid / std::max(1, K)));
+          Ks.assign(std::max(items, 0), K);
         }
-        // the 4-bit hand-off tags (run_pass GPU_FLAGS) repeat every 15 strips: a slot is reused
-        // every GW + 1 strips, which must not be a multiple of 15
-        while (K >= 2 && (K * WG + 1) % 15 == 0) --K;
-        if (getenv("SW_DEBUG_PLAN"))
-          fprintf(stderr, "tmode m=%d long_pairs=%d W=%d t_warps=%d big=%d thr=%.0f steps gangs=%d x %d CTAs\n", m,
-                  n_long, W, t_warps, t.big_strips, t_thr, items, K);
+        if (getenv("SW_DEBUG_PLAN")) {
+          fprintf(stderr, "tmode m=%d long_pairs=%d W=%d t_warps=%d big=%d thr=%.0f steps gangs=%d (CTAs", m,
+                  n_long, W, t_warps, t.big_strips, t_thr, items);
+          for (int i = 0; i < items; ++i) fprintf(stderr, " %d", Ks[i]);
+          fprintf(stderr, ")\n");
+        }
         if (items > 0 && K >= 2) {
           t.gang_items = items;
-          t.gang_ctas = K;
+          t.gang_ctas = K;           // the largest gang (buffer stride); per-gang sizes in gang_base
+          h_gang_base.assign(1, 0);
+          for (int i = 0; i < items; ++i) h_gang_base.push_back(h_gang_base.back() + Ks[i]);
           t.big_strips = 1 << 30;
           // the gang CTAs' other warps wait (measured: letting them stream meanwhile slows the
           // gang's latency-bound strip pipeline more than it gains: C2 query 567 long-only at
@@ -813,7 +827,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     if (t.gang_items > 0) {
       const int GW = t.gang_ctas * t.gang_warps;
       const size_t ints = 1 + 3 * (size_t)t.gang_items + (size_t)t.gang_items * (GW + 1);
-      rc = grow(h, &s.d_gang, &s.gang_cap, ints * sizeof(int32_t), "alloc gang scratch", tst);
+      rc = grow(h, &s.d_gang, &s.gang_cap, (ints + t.gang_items + 1) * sizeof(int32_t), "alloc gang scratch", tst);
       if (rc) return rc;
       const size_t grb_bytes = (size_t)t.gang_items * (GW + 1) * (qcols + kPadCols + 1) * sizeof(uint2);
       rc = grow(h, &s.d_grb, &s.grb_cap, grb_bytes, "alloc gang row buffers", tst, true);
@@ -834,6 +848,10 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
       t.gbest = s.d_gang + 1;
       t.gdone = s.d_gang + 1 + 2 * t.gang_items;
       t.gprog = reinterpret_cast<uint32_t*>(s.d_gang + 1 + 3 * t.gang_items);
+      int32_t* d_base = s.d_gang + ints;   // gang_items + 1 slot offsets (CTAs of gang i: base[i] .. base[i+1])
+      SW_CUDA(h, cudaMemcpyAsync(d_base, h_gang_base.data(), h_gang_base.size() * sizeof(int32_t),
+                                 cudaMemcpyHostToDevice, tst));
+      t.gang_base = d_base;
       t.grb = s.d_grb;
     }
     t.rb = s.d_rb_t;

@@ -1355,20 +1355,21 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
 // two gang launches never hold SMs while waiting for each other.
 template <int C, class CC>
 __device__ __forceinline__ void t_gang_item(const TParams& p, const CC& c, uint8_t* tab, const int8_t* wp,
-                                            int gi, int rank, int warp) {
+                                            int gi, int rank, int K, int warp) {
   using L = LaneS16x2;
   constexpr int CB = chunk_bytes<C>();
   constexpr int LS = 32 * C;
   const int lane = threadIdx.x & 31;
   const int A1 = p.A_used + 1;
   const int qsteps = (p.qcols + 32 + 3) & ~3;
-  const int GW = p.gang_ctas * p.gang_warps;
+  const int GW = K * p.gang_warps;                 // this gang's warps
+  const int GWmax = p.gang_ctas * p.gang_warps;    // buffer stride: the largest gang's slots
   const int gw = rank * p.gang_warps + warp;
   const int ncols = p.pair_ncols[gi];
   const int S = (ncols + LS - 1) / LS;
   const uint16_t* cp = p.cols + p.pair_off[gi];
   // tagged hand-off slots: one 64-bit word per column (run_pass GPU_FLAGS)
-  uint2* rb = p.grb + (int64_t)gi * (GW + 1) * p.rb_cols;
+  uint2* rb = p.grb + (int64_t)gi * (GWmax + 1) * p.rb_cols;
   uint32_t b = 0;
   for (int P = gw; P < S; P += GW) {
     build_strip_tables<C>(p, tab, wp, cp, ncols, P * LS + lane * C);
@@ -1462,18 +1463,22 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
     __shared__ int32_t sgslot;
     if (threadIdx.x == 0) sgslot = atomicAdd(p.gang_ctr, 1);
     __syncthreads();
-    const int gi = sgslot / p.gang_ctas, rank = sgslot % p.gang_ctas;
+    // slot -> (gang, rank): gangs have their own sizes (gang_base prefix of CTAs)
+    int gi = 0;
+    while (gi < p.gang_items && p.gang_base[gi + 1] <= sgslot) ++gi;
+    const int rank = gi < p.gang_items ? sgslot - p.gang_base[gi] : 0;
+    const int K = gi < p.gang_items ? p.gang_base[gi + 1] - p.gang_base[gi] : 0;
     if (gi < p.gang_items) {
       if (p.gang_share) {
         if (warp < p.gang_warps) {
-          t_gang_item<C>(p, c, tab, wp, gi, rank, warp);
+          t_gang_item<C>(p, c, tab, wp, gi, rank, K, warp);
           return;
         }
         wbase = p.gang_warps;
         W = min(W, p.warps - wbase);
         while ((p.warps - wbase) % W) --W;
       } else {
-        if (warp < p.gang_warps) t_gang_item<C>(p, c, tab, wp, gi, rank, warp);
+        if (warp < p.gang_warps) t_gang_item<C>(p, c, tab, wp, gi, rank, K, warp);
         __syncthreads();
       }
     }

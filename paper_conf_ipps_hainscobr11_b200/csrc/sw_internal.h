@@ -135,7 +135,8 @@ struct TParams {
   int A_used;                // popcount(qmask): compact letter k = the k-th set bit; pad = A_used
   // gangs (k_search_t phase 0): pairs [0, gang_items) are spread over gang_ctas CTAs x
   // gang_warps warps each; all buffers below are per gang pair and zeroed before the launch
-  int gang_items, gang_ctas, gang_warps;
+  int gang_items, gang_ctas, gang_warps;   // gang_ctas: the largest gang's CTAs (buffer stride)
+  const int32_t* gang_base;  // gang_items + 1 CTA-slot offsets: gang i has CTAs base[i] .. base[i+1]
   int gang_share;            // 1: the gang CTAs' other warps run the team stream meanwhile
   int gang_chain2;           // 1: the gang warps use the two-op vertical chain (cell_rows CHAIN2)
   int packed;                // team stream layout: 1 packed lanes (mostly short pairs), 0 one pair per strip
