@@ -634,7 +634,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const CC& c,
   // descriptors (len | (P + 1) << 24) of the two newest segments, by segment parity
   gs->desc[0] = (uint32_t)gs->f_len | (1u << 24); gs->desc[1] = 0;
   gs->f_seg = 0;
-  gs->fn = 0;                 // index of the next fetch (= the step at which lane 0 consumes it)
+  gs->fn = 0;                 // MULTI: index of the next fetch, kept in shared memory
   gs->pending = 0;            // a finished pair waits for its cross-lane reduction
   gs->e_pair = 0; gs->e_due = 0;
   gs->nx_pair = -2;           // -2: the next pair is not fetched yet
@@ -643,13 +643,29 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const CC& c,
   // this group's 4 fetches: residues g_cols[k] and top-boundary rows g_rb[k]
   const uint16_t* g_cols;
   const uint2* g_rb;
-  auto plan_group = [&]() {   // warp-uniform
+  // Plain groups: most groups only advance the fetch cursor by 4 positions inside a segment.
+  // plan_group (the full, shared-memory scheduler step) runs for a group that starts a segment,
+  // ends the stream, is due to emit a finished pair, or follows a gap group; it then counts the
+  // plain groups that follow (quiet) and pre-commits the cursor they reach, and the loop
+  // advances g_cols / g_rb in registers for those (ncu on query 5478: the per-group scheduler
+  // was 8.9 % of the warp samples of the step loop).
+  // (measured on C2, T = 3072, one kernel per stream variant (k_search GS): query 729 / 1500
+  // 24.08 / 47.27 -> 23.37 / 45.86 ms; query 5478 over the autotune's candidates R = 44 / 35 /
+  // 45 / 46: 180.4 / 181.1 / 183.9 / 192.3 -> 175.4 / 177.1 / 182.4 / 186.6 ms, R = 43 174.0 ->
+  // 174.9 ms — the step code's register allocation moves by ~1-2 % with any change to the loop)
+  constexpr bool kPlain = true;
+  int quiet = 0;
+  int rb_inc = 0;             // 4 when the plain groups read the previous strip's row buffer
+  // fn: index of the next fetch (= the stream position at which lane 0 consumes it); S: the
+  // stream position of lane 0 at the start of the group (pending emissions are checked then)
+  auto plan_group = [&](int fn, int S) {   // warp-uniform
     int f_pair = gs->f_pair, f_len = gs->f_len, f_P = gs->f_P, f_col = gs->f_col;
     if (f_col == f_len) {     // the next segment starts: this group fetches its gap
       if (f_P + 1 < passes) {
         ++f_P;
       } else {
-        gs->pending = 1; gs->e_pair = f_pair; gs->e_due = gs->fn + 35;
+        // (MULTI reads the fetch index from shared memory: the measured register allocation)
+        gs->pending = 1; gs->e_pair = f_pair; gs->e_due = (MULTI ? gs->fn : fn) + 35;
         __syncwarp();
         if (gs->nx_pair == -2) prefetch();
         if (gs->nx_pair >= 0) {
@@ -679,9 +695,20 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const CC& c,
     } else {
       g_cols = f_cols + (f_col - kGap + 1);
       g_rb = (f_col >= kGap && f_P > 0) ? rb + (f_col - kGap) : p.rb_zero;
+      if constexpr (kPlain) {
+        // the groups after this one fetch f_col + 4, f_col + 8, ... < f_len: plain unless this
+        // is the gap group (the next one switches g_rb from rb_zero to the row buffer) or a
+        // pending emission falls due (the first group with S' >= e_due must run the full step)
+        rb_inc = f_P > 0 ? 4 : 0;
+        quiet = 0;
+        if (f_col >= kGap) {
+          quiet = (f_len - f_col - 4) >> 2;
+          if (gs->pending) quiet = min(quiet, max(0, (gs->e_due - S - 1) >> 2));
+        }
+      }
     }
-    if (f_pair >= 0) gs->f_col = f_col + 4;
-    gs->fn = gs->fn + 4;
+    if (f_pair >= 0) gs->f_col = f_col + 4 + 4 * quiet;
+    if constexpr (MULTI) gs->fn = gs->fn + 4;
     __syncwarp();
   };
   uint32_t ring_res[4], ring_h[4], ring_f[4];
@@ -703,7 +730,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const CC& c,
   const uint8_t* prow = pbase;
   bool store_rb = false;      // lane 31 in a strip whose bottom row feeds the next strip
 
-  plan_group();
+  plan_group(0, -4);
 #pragma unroll
   for (int k = 0; k < 4; ++k) fetch(k);
 
@@ -754,17 +781,23 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const CC& c,
 #pragma unroll
       for (int r = 0; r < R; ++r) { e[r] = nrho; t[r] = 0u; }
     }
-    __syncwarp();
-    if (gs->pending && S >= gs->e_due) {   // every lane has parked the finished pair's maximum
-      uint32_t b = bdone;
+    __syncwarp();   // (also orders lane 31's row-buffer stores before lane 0's later loads)
+    if (kPlain && quiet > 0) {   // plain group (warp-uniform): advance the fetch cursor only
+      --quiet;
+      g_cols += 4;
+      g_rb += rb_inc;
+    } else {
+      if (gs->pending && S >= gs->e_due) {   // every lane has parked the finished pair's maximum
+        uint32_t b = bdone;
 #pragma unroll
-      for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
-      if (lane == 0) emit<L>(p, b, gs->e_pair, 0);
-      __syncwarp();
-      gs->pending = 0;
+        for (int o = 16; o >= 1; o >>= 1) b = L::max2(b, __shfl_xor_sync(SWB_FULL, b, o));
+        if (lane == 0) emit<L>(p, b, gs->e_pair, 0);
+        __syncwarp();
+        gs->pending = 0;
+      }
+      if (gs->f_pair < 0 && !gs->pending) break;
+      plan_group(S + 4, S);   // the 4 fetches issued during this group (consumed in the next one)
     }
-    if (gs->f_pair < 0 && !gs->pending) break;
-    plan_group();   // the 4 fetches issued during this group (consumed in the next one)
     step(std::integral_constant<int, 0>{});
     step(std::integral_constant<int, 1>{});
     step(std::integral_constant<int, 2>{});
@@ -773,7 +806,12 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const CC& c,
   }
 }
 
-template <class L, int G, int Rs, int Rl, int NT, bool WIDE = false>
+// GS: which group-stream variants the kernel contains (G = 32): 0 = both, chosen per launch by
+// p.short_passes; 1 = the single-strip stream only; 2 = the multi-strip stream only.  The
+// launcher compiles and picks 1 / 2 separately, so that each stream loop gets the kernel's
+// registers and instruction cache to itself (the two loops in one kernel shared one register
+// allocation: a change to one moved the other's timing by up to 2 %).
+template <class L, int G, int Rs, int Rl, int NT, bool WIDE = false, int GS = 0>
 __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
   constexpr int kWarps = NT / 32;
   extern __shared__ __align__(128) uint8_t smem[];
@@ -869,8 +907,14 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
       constexpr int CBs = chunk_bytes<Rs>();
       __shared__ GsState sgs[kWarps];
       uint2* rbw = p.rb_group + (int64_t)(blockIdx.x * kWarps + warp) * p.rb_group_cols + 4;
-      if (p.short_passes > 1) group_stream<L, Rs, true>(p, c, smem + p.lg.off + lane * CBs, rbw, &sgs[warp]);
-      else group_stream<L, Rs, false>(p, c, smem + p.lg.off + lane * CBs, rbw, &sgs[warp]);
+      if constexpr (GS == 2) {
+        group_stream<L, Rs, true>(p, c, smem + p.lg.off + lane * CBs, rbw, &sgs[warp]);
+      } else if constexpr (GS == 1) {
+        group_stream<L, Rs, false>(p, c, smem + p.lg.off + lane * CBs, rbw, &sgs[warp]);
+      } else {
+        if (p.short_passes > 1) group_stream<L, Rs, true>(p, c, smem + p.lg.off + lane * CBs, rbw, &sgs[warp]);
+        else group_stream<L, Rs, false>(p, c, smem + p.lg.off + lane * CBs, rbw, &sgs[warp]);
+      }
       return;
     }
   }
@@ -1517,19 +1561,40 @@ cudaError_t configure_tmode(int smem_bytes, int* blocks_per_sm) {
                                                        smem_bytes);
 }
 
+// G = 32 entries compile two kernels (GS = 1: single-strip group stream, GS = 2: multi-strip);
+// the 32-bit recompute (item_list) never reaches the group phase, so either serves it.
 template <class L, int G, int Rs, int Rl, int NT, bool WIDE>
 cudaError_t launch_search_t(const SearchParams& p, int grid, int smem_bytes, cudaStream_t st) {
-  k_search<L, G, Rs, Rl, NT, WIDE><<<grid, NT, smem_bytes, st>>>(p);
+  if constexpr (G == 32) {
+    if (p.short_passes > 1) k_search<L, G, Rs, Rl, NT, WIDE, 2><<<grid, NT, smem_bytes, st>>>(p);
+    else k_search<L, G, Rs, Rl, NT, WIDE, 1><<<grid, NT, smem_bytes, st>>>(p);
+  } else {
+    k_search<L, G, Rs, Rl, NT, WIDE><<<grid, NT, smem_bytes, st>>>(p);
+  }
   return cudaGetLastError();
+}
+
+template <class L, int G, int Rs, int Rl, int NT, bool WIDE, int GS>
+cudaError_t configure_one(int smem_bytes, int* blocks_per_sm) {
+  cudaError_t e = cudaFuncSetAttribute(k_search<L, G, Rs, Rl, NT, WIDE, GS>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+  if (e != cudaSuccess) return e;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search<L, G, Rs, Rl, NT, WIDE, GS>, NT,
+                                                       smem_bytes);
 }
 
 template <class L, int G, int Rs, int Rl, int NT, bool WIDE>
 cudaError_t configure_t(int smem_bytes, int* blocks_per_sm) {
-  cudaError_t e = cudaFuncSetAttribute(k_search<L, G, Rs, Rl, NT, WIDE>,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
-  if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search<L, G, Rs, Rl, NT, WIDE>, NT,
-                                                       smem_bytes);
+  if constexpr (G == 32) {
+    int b1 = 0, b2 = 0;
+    cudaError_t e = configure_one<L, G, Rs, Rl, NT, WIDE, 1>(smem_bytes, &b1);
+    if (e != cudaSuccess) return e;
+    e = configure_one<L, G, Rs, Rl, NT, WIDE, 2>(smem_bytes, &b2);
+    *blocks_per_sm = b1 < b2 ? b1 : b2;
+    return e;
+  } else {
+    return configure_one<L, G, Rs, Rl, NT, WIDE, 0>(smem_bytes, blocks_per_sm);
+  }
 }
 
 }  // namespace swb

@@ -18,6 +18,8 @@ T = int(sys.argv[2]) if len(sys.argv) > 2 else 3072
 reps = int(sys.argv[3]) if len(sys.argv) > 3 else 2
 cfg = sys.argv[4] if len(sys.argv) > 4 else "C2"
 q = gen.make_query(L)
+if os.environ.get("SW_LIB"):          # A/B against another build of the library
+    swp.load_library(os.environ["SW_LIB"])
 if cfg == "C3":
     lens = gen.long_lengths(4096, seed=3)
     db = gen.build_database(lens, 3, [q])
