@@ -586,7 +586,7 @@ __device__ __forceinline__ void emit(const SearchParams& p, uint32_t b, int pair
 struct GsState {
   int64_t f_off;    // column offset of the pair being fetched (u16 units)
   int64_t nx_off;   // prefetched next pair's column offset
-  int f_pair, f_len, f_P, f_col, f_seg, fn;
+  int f_pair, f_len, f_P, f_col, f_seg;
   int nx_pair, nx_len;
   int pending, e_pair, e_due;
   uint32_t desc[2];
@@ -634,7 +634,6 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const CC& c,
   // descriptors (len | (P + 1) << 24) of the two newest segments, by segment parity
   gs->desc[0] = (uint32_t)gs->f_len | (1u << 24); gs->desc[1] = 0;
   gs->f_seg = 0;
-  gs->fn = 0;                 // MULTI: index of the next fetch, kept in shared memory
   gs->pending = 0;            // a finished pair waits for its cross-lane reduction
   gs->e_pair = 0; gs->e_due = 0;
   gs->nx_pair = -2;           // -2: the next pair is not fetched yet
@@ -664,8 +663,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const CC& c,
       if (f_P + 1 < passes) {
         ++f_P;
       } else {
-        // (MULTI reads the fetch index from shared memory: the measured register allocation)
-        gs->pending = 1; gs->e_pair = f_pair; gs->e_due = (MULTI ? gs->fn : fn) + 35;
+        gs->pending = 1; gs->e_pair = f_pair; gs->e_due = fn + 35;
         __syncwarp();
         if (gs->nx_pair == -2) prefetch();
         if (gs->nx_pair >= 0) {
@@ -708,7 +706,6 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const CC& c,
       }
     }
     if (f_pair >= 0) gs->f_col = f_col + 4 + 4 * quiet;
-    if constexpr (MULTI) gs->fn = gs->fn + 4;
     __syncwarp();
   };
   uint32_t ring_res[4], ring_h[4], ring_f[4];
