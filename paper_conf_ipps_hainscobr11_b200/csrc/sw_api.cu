@@ -45,6 +45,9 @@ struct QuerySlot {
   size_t grb_cap = 0;
   cudaStream_t stream = nullptr;
   cudaStream_t aux = nullptr;      // T-mode launch, concurrent with the group launch
+  cudaStream_t scan = nullptr;     // row-scan cluster launches (sw_scan.cu), beside the T-mode launch
+  cudaEvent_t scan_fork = nullptr, scan_done = nullptr;
+  int scan_smem = -1;              // the row-scan kernel's configured dynamic shared memory
   cudaEvent_t done = nullptr;
   cudaEvent_t fork = nullptr, join = nullptr;
 };
@@ -373,6 +376,14 @@ int ensure_slots(sw_handle h, int n) {
     QuerySlot s;
     SW_CUDA(h, cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking));
     SW_CUDA(h, cudaStreamCreateWithFlags(&s.aux, cudaStreamNonBlocking));
+    {   // the row-scan clusters must be placed before the T-mode kernel's persistent CTAs fill the
+        // GPU (launched first on their own stream, but only priority makes the order hold)
+      int lo = 0, hi = 0;
+      SW_CUDA(h, cudaDeviceGetStreamPriorityRange(&lo, &hi));
+      SW_CUDA(h, cudaStreamCreateWithPriority(&s.scan, cudaStreamNonBlocking, hi));
+    }
+    SW_CUDA(h, cudaEventCreateWithFlags(&s.scan_fork, cudaEventDisableTiming));
+    SW_CUDA(h, cudaEventCreateWithFlags(&s.scan_done, cudaEventDisableTiming));
     SW_CUDA(h, cudaEventCreateWithFlags(&s.fork, cudaEventDisableTiming));
     SW_CUDA(h, cudaEventCreateWithFlags(&s.join, cudaEventDisableTiming));
     SW_CUDA(h, cudaEventCreateWithFlags(&s.done, cudaEventDisableTiming));
@@ -676,6 +687,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     }
     TParams t{};
     std::vector<int32_t> h_gang_base;   // per-gang CTA slot offsets (uploaded with the gang scratch)
+    std::vector<int> scan_cols;         // row-scan items [0, size): columns per CTA
     t.matrix = h->d_matrix;
     t.A = h->A;
     t.rho = h->rho16;
@@ -764,6 +776,38 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
         t_thr /= nw;
         const bool hidden = (double)sp.short_cols > 0.5 * (double)sp.long_cols;
         int K = 0, items = 0;
+        // Row scan (sw_scan.cu): the longest pairs of a launch
+        // that is not hidden run one query row per cluster time step instead of strip pipelines
+        // (their wavefront bound): a prefix of the long pairs (longest first) with at least
+        // kScanMinCols columns and at most kScanCtas x kScanCols, each on a cluster of kScanCtas
+        // CTAs, all in one launch.  SW_SCAN=0 disables it, SW_SCAN=N forces it for every
+        // long pair of >= N columns (tests, probes).
+        {
+          int scan_min = kScanMinCols;
+          bool forced = false;
+          if (const char* f = getenv("SW_SCAN"); f && *f) { scan_min = atoi(f); forced = scan_min > 0; }
+          if (scan_min > 0 && (forced || !hidden) && !h->wide && a_used + 1 <= kScanMaxLetters) {
+            for (int pp = 0; pp < n_long && pp < (forced ? 4 : kMaxScanItems); ++pp) {
+              const int nc = h->db->h_pair_ncols[pp];
+              if (nc < scan_min || nc > kScanCtas * kScanCols) break;
+              if (!forced) {
+                // only an outlier: a pair whose time alone bounds the launch (a gang candidate)
+                // AND is >= 1.5x the next pair's columns.  The scan computes ~2.7x fewer cells
+                // per SM than the team stream (C2 top pair, query 567: 0.418 ms on 16 SMs vs
+                // 0.693 ms as a gang), so for a tail of similar pairs (C2 at T = 3072: 22 pairs
+                // of 16-35k columns) it only takes SMs from the others: 0.98 vs 0.92 ms
+                const double S = std::ceil((double)nc / spos);
+                if (item_time(S >= t.big_strips ? t_warps : W, S) <= 1.15 * t_thr) break;
+                if (pp + 1 < n_long && nc < 1.5 * h->db->h_pair_ncols[pp + 1]) break;
+              }
+              scan_cols.push_back(scan_cols_cta(nc, kScanCtas));
+            }
+          }
+          if (getenv("SW_DEBUG_PLAN") && !scan_cols.empty())
+            fprintf(stderr, "tmode scan items=%zu (first %d columns per CTA)\n", scan_cols.size(), scan_cols[0]);
+        }
+        // gangs for the long pairs after the scanned ones (gang gi = pair scan items + gi)
+        const int s0 = (int)scan_cols.size();
         std::vector<int> Ks;   // CTAs of each gang (the longest pairs need more than the others)
         if (!hidden) {
           // a gang of GW warps: each warp runs ceil(S / GW) strips back to back after a ramp of
@@ -774,7 +818,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
             return std::max(std::ceil(S / GW) * qsteps + (std::min<double>(GW, S) - 1.0) * lag,
                             (S - 1.0) * lag + qsteps);
           };
-          for (int pp = 0; pp < n_long && pp < kMaxGangItems; ++pp) {
+          for (int pp = s0; pp < n_long && pp - s0 < kMaxGangItems; ++pp) {
             const double S = std::ceil((double)h->db->h_pair_ncols[pp] / spos);
             const double alone = item_time(S >= t.big_strips ? t_warps : W, S);
             if (alone <= 1.15 * t_thr || S < 2.0 * W) break;
@@ -801,7 +845,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
           while (K >= 2 && (K * WG + 1) % 15 == 0) --K;
           const char* comma = strchr(f, ':');
           items = comma ? atoi(comma + 1) : n_long;
-          items = std::min(items, std::min(n_long, t_grid / std::max(1, K)));
+          items = std::min(items, std::min(n_long - s0, t_grid / std::max(1, K)));
           Ks.assign(std::max(items, 0), K);
         }
         if (getenv("SW_DEBUG_PLAN")) {
@@ -824,6 +868,8 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
         }
       }
     }
+    t.gang0 = (int)scan_cols.size();
+    t.q0 = t.gang0 + t.gang_items;
     if (t.gang_items > 0) {
       const int GW = t.gang_ctas * t.gang_warps;
       const size_t ints = 1 + 3 * (size_t)t.gang_items + (size_t)t.gang_items * (GW + 1);
@@ -860,7 +906,23 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     t.packed = t_packed;
     if (t.gang_items > 0) SW_CUDA(h, cudaStreamWaitEvent(tst, h->gang_ev, 0));
     SW_CUDA(h, cudaEventRecord(ev[3], tst));
-    SW_CUDA(h, launch_tmode(t, t_grid, t_smem, tst));
+    if (!scan_cols.empty()) {
+      // the row-scan clusters go first on the T-mode stream and the T-mode kernel follows as a
+      // programmatic dependent launch (the scan kernel triggers once its clusters are resident):
+      // launched on another stream, the T-mode kernel's persistent CTAs could take every SM
+      // first and leave no GPC free for a 16-CTA cluster until they finish (measured: the two
+      // kernels serialised).  The T-mode queue starts after the scanned pairs (t.q0).
+      const int ssmem = scan_smem_bytes(a_used, scan_cols[0], qcols);
+      if (s.scan_smem != ssmem) {
+        int maxc = 0;
+        cudaError_t e = configure_scan_kernel(ssmem, kScanCtas, &maxc);
+        if (e != cudaSuccess) return cuda_fail(h, e, "configure row-scan kernel");
+        if (maxc < 1) return fail(h, SW_E_UNSUPPORTED, "row-scan cluster cannot be placed");
+        s.scan_smem = ssmem;
+      }
+      SW_CUDA(h, launch_scan_pairs(t, (int)scan_cols.size(), kScanCtas, ssmem, tst));
+    }
+    SW_CUDA(h, launch_tmode(t, t_grid, t_smem, tst, false, !scan_cols.empty()));
     SW_CUDA(h, cudaEventRecord(ev[4], tst));
     if (t.gang_items > 0) SW_CUDA(h, cudaEventRecord(h->gang_ev, tst));
     if (t.dbg_times) {   // probe output: strip P start / end relative to strip 0's start (us)
@@ -885,6 +947,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
       r.item_count = s.d_ovf_count;
       r.work = s.d_work + 2;
       r.gang_items = 0;
+      r.q0 = 0;
       r.big_strips = 1 << 30;
       r.team_warps = std::min(2, t.warps);
       while (t.warps % r.team_warps) --r.team_warps;
@@ -1624,6 +1687,9 @@ void sw_destroy(sw_handle h) {
     cudaFree(s.d_gang); cudaFree(s.d_grb);
     if (s.stream) cudaStreamDestroy(s.stream);
     if (s.aux) { cudaStreamSynchronize(s.aux); cudaStreamDestroy(s.aux); }
+    if (s.scan) { cudaStreamSynchronize(s.scan); cudaStreamDestroy(s.scan); }
+    if (s.scan_fork) cudaEventDestroy(s.scan_fork);
+    if (s.scan_done) cudaEventDestroy(s.scan_done);
     if (s.fork) cudaEventDestroy(s.fork);
     if (s.join) cudaEventDestroy(s.join);
     if (s.done) cudaEventDestroy(s.done);

@@ -1031,7 +1031,8 @@ __device__ __forceinline__ void emit_t32(const TParams& p, int score, int sq) { 
 // an item already taken for this team (or -1).  min_strips: a team of W warps only keeps items
 // with at least this many strips (fewer: the item is parked in *parked and the loop returns,
 // so that the CTA can regroup into smaller teams for the remaining, shorter items).  Items
-// [0, gang_items) belong to the gangs (t_gang_item); the queue starts after them.
+// [0, gang_items) belong to the gangs (t_gang_item), [0, q0) to the gangs or the row-scan
+// launches (sw_scan.cu); the queue starts at q0.
 template <int C, class CC>
 __device__ __forceinline__ void t_team_loop(const TParams& p, const CC& c, uint8_t* tab,
                                             const int8_t* wp, int W, int team, int wt, int first_item,
@@ -1047,7 +1048,7 @@ __device__ __forceinline__ void t_team_loop(const TParams& p, const CC& c, uint8
   for (;;) {
     team_bar(team, W);
     if (wt == 0 && lane == 0) {
-      const int it = pending >= 0 ? pending : p.gang_items + atomicAdd(p.work, 1);
+      const int it = pending >= 0 ? pending : p.q0 + atomicAdd(p.work, 1);
       sitem[team] = it;
       for (int i = 0; i <= W; ++i) prog[i] = 0u;
     }
@@ -1167,7 +1168,7 @@ __device__ __forceinline__ void t_team_stream_pairs(const TParams& p, const CC& 
         if (vs->end) break;
         if (atomicCAS(&ts->lock, 0, 1) == 0) {
           while (vs->next <= g && !vs->end) {
-            const int item = p.gang_items + atomicAdd(p.work, 1);
+            const int item = p.q0 + atomicAdd(p.work, 1);
             if (item >= n_items) { vs->end = 1; break; }
             append(item);
           }
@@ -1288,14 +1289,14 @@ __device__ __forceinline__ void t_team_stream(const TParams& p, const CC& c, uin
   // longest first, so the length of the item at the counter tells which case applies)
   auto take = [&]() -> int {
     if (vs->pend == vs->pend_end) {
-      const int cur = *reinterpret_cast<volatile int*>(p.work) + p.gang_items;
+      const int cur = *reinterpret_cast<volatile int*>(p.work) + p.q0;
       int hf = 0;
       const bool short_pairs = cur < n_items && p.pair_ncols[pair_of(cur, &hf)] < 32 * C;
       const int grab = short_pairs ? kTGrab : 1;
       const int b0 = atomicAdd(p.work, grab);
       vs->pend = b0; vs->pend_end = b0 + grab;
     }
-    const int item = p.gang_items + vs->pend;
+    const int item = p.q0 + vs->pend;
     vs->pend = vs->pend + 1;
     return item < n_items ? item : -1;
   };
@@ -1406,9 +1407,10 @@ __device__ __forceinline__ void t_gang_item(const TParams& p, const CC& c, uint8
   const int GW = K * p.gang_warps;                 // this gang's warps
   const int GWmax = p.gang_ctas * p.gang_warps;    // buffer stride: the largest gang's slots
   const int gw = rank * p.gang_warps + warp;
-  const int ncols = p.pair_ncols[gi];
+  const int item = p.gang0 + gi;                   // the pair (gi indexes the gang buffers)
+  const int ncols = p.pair_ncols[item];
   const int S = (ncols + LS - 1) / LS;
-  const uint16_t* cp = p.cols + p.pair_off[gi];
+  const uint16_t* cp = p.cols + p.pair_off[item];
   // tagged hand-off slots: one 64-bit word per column (run_pass GPU_FLAGS)
   uint2* rb = p.grb + (int64_t)gi * (GWmax + 1) * p.rb_cols;
   uint32_t b = 0;
@@ -1444,7 +1446,7 @@ __device__ __forceinline__ void t_gang_item(const TParams& p, const CC& c, uint8
     if (atomicAdd(&p.gdone[gi], 1) == GW - 1) {   // the last warp of the gang
       __threadfence();
       const int lo = atomicAdd(&p.gbest[2 * gi], 0), hi = atomicAdd(&p.gbest[2 * gi + 1], 0);
-      emit_t(p, ((uint32_t)lo & 0xffffu) | ((uint32_t)hi << 16), gi);
+      emit_t(p, ((uint32_t)lo & 0xffffu) | ((uint32_t)hi << 16), item);
     }
   }
 }
@@ -1543,10 +1545,25 @@ __global__ void __launch_bounds__(NT, 1) k_search_t(const TParams p) {
   }
 }
 
+// pdl: programmatic dependent launch after the row-scan kernel on the same stream (its
+// clusters are resident and have triggered before these CTAs fill the remaining SMs)
 template <int C, int NT, bool WIDE, class L, bool PACKED>
-cudaError_t launch_search_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st) {
-  k_search_t<C, NT, WIDE, L, PACKED><<<grid, NT, smem_bytes, st>>>(p);
-  return cudaGetLastError();
+cudaError_t launch_search_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st, bool pdl = false) {
+  if (!pdl) {
+    k_search_t<C, NT, WIDE, L, PACKED><<<grid, NT, smem_bytes, st>>>(p);
+    return cudaGetLastError();
+  }
+  cudaLaunchConfig_t cfg = {};
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(NT);
+  cfg.dynamicSmemBytes = smem_bytes;
+  cfg.stream = st;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, k_search_t<C, NT, WIDE, L, PACKED>, p);
 }
 
 template <int C, int NT, bool WIDE, class L, bool PACKED>

@@ -136,6 +136,9 @@ struct TParams {
   // gangs (k_search_t phase 0): pairs [0, gang_items) are spread over gang_ctas CTAs x
   // gang_warps warps each; all buffers below are per gang pair and zeroed before the launch
   int gang_items, gang_ctas, gang_warps;   // gang_ctas: the largest gang's CTAs (buffer stride)
+  int gang0;                 // first gang pair: gang gi works on pair gang0 + gi (after the
+                             // row-scan pairs [0, gang0), sw_scan.cu)
+  int q0;                    // first item of the team queue: gang0 + gang_items
   const int32_t* gang_base;  // gang_items + 1 CTA-slot offsets: gang i has CTAs base[i] .. base[i+1]
   int gang_share;            // 1: the gang CTAs' other warps run the team stream meanwhile
   int gang_chain2;           // 1: the gang warps use the two-op vertical chain (cell_rows CHAIN2)
@@ -149,10 +152,26 @@ struct TParams {
   int32_t* gdone;            // gang_items: warps finished
 };
 
-cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st, bool s32 = false);
+cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st, bool s32 = false,
+                         bool pdl = false);
 cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm, bool wide, bool s32 = false,
                                    bool packed = false);
 cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, uint32_t qmask, cudaStream_t st);
+
+// Row scan (sw_scan.cu): long pairs [0, items) on one cluster of `ctas` CTAs each (one launch),
+// ceil(ncols / ctas) columns per CTA rounded up to 128 (<= kScanCols); the scores are emitted
+// like k_search_t's (emit_t).
+constexpr int kScanThreads = 1024;
+constexpr int kScanC = 4;
+constexpr int kScanCols = kScanThreads * kScanC;
+constexpr int kScanCtas = 16;            // cluster size (non-portable, <= 16)
+constexpr int kScanMaxLetters = 26;      // (A_used + 1) x 2 x cols_cta bytes of tables + the query
+constexpr int kScanMinCols = 16384;      // pairs from 1024 columns per CTA up
+constexpr int kMaxScanItems = 1;      // each takes 16 SMs from the team stream (C2 query 567, T = 3072: 4 items 1.32 ms, 1 item see DESIGN)
+int scan_cols_cta(int ncols, int ctas);
+int scan_smem_bytes(int a_used, int cols_cta, int qcols);
+cudaError_t configure_scan_kernel(int smem_bytes, int ctas, int* max_clusters);
+cudaError_t launch_scan_pairs(const TParams& p, int items, int ctas, int smem_bytes, cudaStream_t st);
 
 // Traceback of one pair (sw_traceback.cu): dir = m*n bytes, scratch = 7*m ints, result = 6 ints.
 cudaError_t launch_traceback(const uint8_t* q, int m, const uint16_t* dcols, int half, int n, const int8_t* W, int A,

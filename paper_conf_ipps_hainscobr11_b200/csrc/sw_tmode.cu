@@ -24,9 +24,9 @@ cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, uint32_t
 // s32 = true: the 32-bit recompute of the flagged sequences (p.item_list / p.item_count);
 // p.packed selects the team stream's layout, p.delta > 0 the WIDE instantiation
 template <bool WIDE, class L>
-static cudaError_t launch_t(const TParams& p, int grid, int smem_bytes, cudaStream_t st) {
-  if (p.packed) return launch_search_tmode<kTmodeC, kTmodeThreads, WIDE, L, true>(p, grid, smem_bytes, st);
-  return launch_search_tmode<kTmodeC, kTmodeThreads, WIDE, L, false>(p, grid, smem_bytes, st);
+static cudaError_t launch_t(const TParams& p, int grid, int smem_bytes, cudaStream_t st, bool pdl) {
+  if (p.packed) return launch_search_tmode<kTmodeC, kTmodeThreads, WIDE, L, true>(p, grid, smem_bytes, st, pdl);
+  return launch_search_tmode<kTmodeC, kTmodeThreads, WIDE, L, false>(p, grid, smem_bytes, st, pdl);
 }
 template <bool WIDE, class L>
 static cudaError_t configure_t2(int smem_bytes, int* blocks_per_sm, bool packed) {
@@ -34,9 +34,11 @@ static cudaError_t configure_t2(int smem_bytes, int* blocks_per_sm, bool packed)
   return configure_tmode<kTmodeC, kTmodeThreads, WIDE, L, false>(smem_bytes, blocks_per_sm);
 }
 
-cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st, bool s32) {
-  if (s32) return p.delta > 0 ? launch_t<true, LaneS32>(p, grid, smem_bytes, st) : launch_t<false, LaneS32>(p, grid, smem_bytes, st);
-  return p.delta > 0 ? launch_t<true, LaneS16x2>(p, grid, smem_bytes, st) : launch_t<false, LaneS16x2>(p, grid, smem_bytes, st);
+cudaError_t launch_tmode(const TParams& p, int grid, int smem_bytes, cudaStream_t st, bool s32, bool pdl) {
+  if (s32) return p.delta > 0 ? launch_t<true, LaneS32>(p, grid, smem_bytes, st, pdl)
+                              : launch_t<false, LaneS32>(p, grid, smem_bytes, st, pdl);
+  return p.delta > 0 ? launch_t<true, LaneS16x2>(p, grid, smem_bytes, st, pdl)
+                     : launch_t<false, LaneS16x2>(p, grid, smem_bytes, st, pdl);
 }
 
 cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm, bool wide, bool s32, bool packed) {

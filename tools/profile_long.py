@@ -33,6 +33,12 @@ if len(sys.argv) > 6 and sys.argv[6]:
     idx = np.sort(order[:int(k)] if mode == "top" else order[int(k):])
 off = np.concatenate([[0], np.cumsum(L[idx])]).astype(np.int64)
 res = np.concatenate([db.residues[db.offsets[i]:db.offsets[i + 1]] for i in idx])
+if os.environ.get("SW_PROBE_EXTRA"):   # extra synthetic sequences (e.g. an outlier pair for the row scan)
+    ext = [int(x) for x in os.environ["SW_PROBE_EXTRA"].split(",")]
+    rng = np.random.default_rng(11)
+    res = np.concatenate([res] + [rng.integers(0, 20, size=n).astype(np.uint8) for n in ext])
+    off = np.concatenate([off, off[-1] + np.cumsum(ext)]).astype(np.int64)
+    idx = np.concatenate([idx, np.zeros(len(ext), np.int64)])
 q = gen.make_query(m)
 if os.environ.get("SW_LIB"):          # A/B against another build of the library
     swp.load_library(os.environ["SW_LIB"])

@@ -1,0 +1,8 @@
+mkdir -p gpurun_out/s1
+timeout 600 python -m pytest tests/test_scan_gpu.py -x -q -p no:cacheprovider 2>&1 | tail -3
+for T in 3072 2572 2072 1572; do
+  for sc in 0 ""; do
+    SW_DEBUG_PLAN=1 SW_SCAN=$sc timeout 120 python tools/profile_long.py 567 $T 3 C2 2>&1 | grep -E "scan|GCUPS" | tail -2 | sed "s/^/[scan=$sc] /"
+  done
+done > gpurun_out/s1/long.txt 2>&1
+cat gpurun_out/s1/long.txt
