@@ -172,9 +172,12 @@ int sw_last_regime_ms(sw_handle h, double out[3]);
 
 /* Optimal local alignment of the handle's query with database sequence seq_index (caller
  * order) — the traceback step after the search ("The optimal
- * alignment can be found by backtracking through H").  Computed on the device: an anti-
- * diagonal sweep of Eq.(1) writing one direction byte per cell (m*n bytes of device scratch),
- * then a walk back from the first maximal cell.  Query rows [q_begin, q_end) are aligned to
+ * alignment can be found by backtracking through H").  Computed on the device in bounded
+ * memory: an anti-diagonal sweep of Eq.(1) for the score and the end cell (O(m) scratch), a
+ * sweep of the reversed prefixes anchored at the end cell for the start cell, then a sweep of
+ * the alignment's bounding box only, writing one direction byte per cell ((q_end - q_begin) x
+ * (d_end - d_begin) bytes of device scratch instead of m*n), and a walk back from the first
+ * maximal cell of the box.  Query rows [q_begin, q_end) are aligned to
  * database columns [d_begin, d_end) (0-based, end exclusive; all 0 when score == 0).
  * ops[0 .. n_ops): runs (length << 2) | op, op 0 = M (q_i against d_j), 1 = I (d_j against a
  * gap), 2 = D (q_i against a gap); a gap closed and reopened (possible when sigma > rho) is two
@@ -188,6 +191,14 @@ typedef struct {
   int32_t n_ops;
 } sw_alignment;
 int sw_align(sw_handle h, int64_t seq_index, sw_alignment* out, uint32_t* ops, int32_t ops_cap);
+
+/* The top hits of a score array ("traceback for top hits"): the k largest of
+ * scores[0 .. n) (host array, e.g. sw_search's output), ties broken by the smaller index,
+ * selected on the device (radix-select histograms over the 32-bit keys, then the < k + ties
+ * candidates ordered).  idx_out / score_out (host, min(k, n) entries) receive them best first.
+ * k <= 0 or n == 0: nothing.  Returns SW_E_INVALID for NULL buffers with k > 0 and n > 0.
+ * Blocking.  The handle's stream resources are used; no database is needed. */
+int sw_top_hits(sw_handle h, const int32_t* scores, int64_t n, int32_t k, int64_t* idx_out, int32_t* score_out);
 
 /* Free everything (NULL-safe). */
 void sw_destroy(sw_handle h);

@@ -23,7 +23,7 @@ SW_OK, SW_E_INVALID, SW_E_STATE, SW_E_NOMEM, SW_E_CUDA, SW_E_UNSUPPORTED = range
 SW_AUTO_THRESHOLD = -1
 EXPORTED = ["sw_create", "sw_set_query", "sw_load_db", "sw_search", "sw_search_async",
             "sw_search_batch", "sw_search_batch_async", "sw_search_stream", "sw_last_stats", "sw_last_kernel_ms", "sw_last_regime_ms", "sw_last_threshold",
-            "sw_align", "sw_destroy",
+            "sw_align", "sw_top_hits", "sw_destroy",
             "sw_strerror", "sw_last_error", "sw_version"]
 
 _lib = None
@@ -58,6 +58,8 @@ def load_library(path: str = LIB_PATH):
     L.sw_last_threshold.argtypes = [vp]
     L.sw_align.argtypes = [vp, i64, vp, vp, i32]
     L.sw_align.restype = ctypes.c_int
+    L.sw_top_hits.argtypes = [vp, vp, i64, i32, vp, vp]
+    L.sw_top_hits.restype = ctypes.c_int
     L.sw_last_threshold.restype = ctypes.c_int32
     L.sw_destroy.argtypes = [vp]
     L.sw_destroy.restype = None
@@ -207,6 +209,17 @@ def sw_align(h, seq_index: int, ops_cap: int = 1 << 16) -> dict:
             "d_end": out.d_end, "runs": runs, "cigar": "".join(f"{n}{o}" for o, n in runs)}
 
 
+def sw_top_hits(h, scores, k: int):
+    """The k best (index, score) of a score array, best first (ties: smaller index), selected
+    on the device."""
+    sc = np.ascontiguousarray(scores, dtype=np.int32).reshape(-1)
+    kk = max(0, min(int(k), sc.size))
+    idx = np.zeros(max(kk, 1), dtype=np.int64)
+    val = np.zeros(max(kk, 1), dtype=np.int32)
+    _check(h, load_library().sw_top_hits(h, sc.ctypes.data, sc.size, int(k), idx.ctypes.data, val.ctypes.data))
+    return idx[:kk], val[:kk]
+
+
 def sw_destroy(h):
     if h:
         load_library().sw_destroy(h)
@@ -250,6 +263,9 @@ class SmithWaterman:
 
     def align(self, seq_index: int) -> dict:
         return sw_align(self.h, seq_index)
+
+    def top_hits(self, scores, k: int):
+        return sw_top_hits(self.h, scores, k)
 
     def last_threshold(self) -> int:
         return int(load_library().sw_last_threshold(self.h))

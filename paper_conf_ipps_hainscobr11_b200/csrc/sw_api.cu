@@ -129,6 +129,7 @@ struct sw_handle_s {
   int* d_tb_scratch = nullptr; size_t tb_scratch_cap = 0;
   int* d_tb_result = nullptr; size_t tb_result_cap = 0;
   uint32_t* d_tb_ops = nullptr; size_t tb_ops_cap = 0;
+  uint8_t* d_tk = nullptr; size_t tk_cap = 0;         // sw_top_hits scratch
   uint8_t* d_tb_query = nullptr; size_t tb_query_cap = 0;
   KernelConfig last_cfg{};
   int32_t last_threshold = 0;
@@ -1615,34 +1616,107 @@ int sw_align(sw_handle h, int64_t seq_index, sw_alignment* out, uint32_t* ops, i
   const int64_t n = h->db->sorted_len[(size_t)pos];
   const int m = (int)h->query.size();
   if (n == 0) { out->q_begin = out->q_end = out->d_begin = out->d_end = 0; return SW_OK; }
-  const int64_t cells = (int64_t)m * n;
-  int rc = grow(h, &h->d_tb_dir, &h->tb_dir_cap, (size_t)cells, "alloc traceback directions");
+  int rc = grow(h, &h->d_tb_scratch, &h->tb_scratch_cap, (size_t)7 * m * sizeof(int), "alloc traceback scratch");
   if (rc) return rc;
-  rc = grow(h, &h->d_tb_scratch, &h->tb_scratch_cap, (size_t)7 * m * sizeof(int), "alloc traceback scratch");
-  if (rc) return rc;
-  rc = grow(h, &h->d_tb_result, &h->tb_result_cap, 8 * sizeof(int), "alloc traceback result");
-  if (rc) return rc;
-  const int cap_dev = std::max(1, (int)std::min<int64_t>(m + n, 1 << 24));
-  rc = grow(h, &h->d_tb_ops, &h->tb_ops_cap, (size_t)cap_dev * sizeof(uint32_t), "alloc traceback ops");
+  rc = grow(h, &h->d_tb_result, &h->tb_result_cap, 16 * sizeof(int), "alloc traceback result");
   if (rc) return rc;
   rc = grow(h, &h->d_tb_query, &h->tb_query_cap, (size_t)m, "alloc traceback query");
   if (rc) return rc;
   SW_CUDA(h, cudaMemcpy(h->d_tb_query, h->query.data(), (size_t)m, cudaMemcpyHostToDevice));
   const int64_t pair = pos >> 1;
   const int half = (int)(pos & 1);
-  SW_CUDA(h, launch_traceback(h->d_tb_query, m, h->db->d_cols + h->db->h_pair_off[(size_t)pair], half, (int)n, h->d_matrix,
-                              h->A, h->rho32, h->sigma32, h->d_tb_dir, h->d_tb_scratch, h->d_tb_result, h->d_tb_ops,
-                              cap_dev, nullptr));
+  const uint16_t* dcols = h->db->d_cols + h->db->h_pair_off[(size_t)pair];
+  // (1) score and end cell, (2) start cell — O(m) scratch (sw_traceback.cu)
+  SW_CUDA(h, launch_tb_score_start(h->d_tb_query, m, dcols, half, (int)n, h->d_matrix, h->A, h->rho32, h->sigma32,
+                                   h->d_tb_scratch, h->d_tb_result, nullptr));
+  int se[5];
+  SW_CUDA(h, cudaMemcpy(se, h->d_tb_result, sizeof(se), cudaMemcpyDeviceToHost));
+  out->score = se[0];
+  if (se[0] <= 0) { out->n_ops = 0; return SW_OK; }
+  const int ib = se[3], jb = se[4], ie = se[1], je = se[2];
+  if (ib < 0 || jb < 0 || ib > ie || jb > je) return fail(h, SW_E_CUDA, "traceback: no start cell found");
+  // (3) directions for the alignment's bounding box only, then the walk
+  const int mb = ie - ib + 1, nb = je - jb + 1;
+  rc = grow(h, &h->d_tb_dir, &h->tb_dir_cap, (size_t)mb * (size_t)nb, "alloc traceback directions");
+  if (rc) return rc;
+  const int cap_dev = std::max(1, mb + nb);
+  rc = grow(h, &h->d_tb_ops, &h->tb_ops_cap, (size_t)cap_dev * sizeof(uint32_t), "alloc traceback ops");
+  if (rc) return rc;
+  SW_CUDA(h, launch_traceback(h->d_tb_query + ib, mb, dcols + jb, half, nb, h->d_matrix, h->A, h->rho32, h->sigma32,
+                              h->d_tb_dir, h->d_tb_scratch, h->d_tb_result + 8, h->d_tb_ops, cap_dev, nullptr));
   int res[6];
-  SW_CUDA(h, cudaMemcpy(res, h->d_tb_result, sizeof(res), cudaMemcpyDeviceToHost));
-  out->score = res[0];
-  if (res[0] > 0) {
-    out->q_begin = res[3]; out->d_begin = res[4];
-    out->q_end = res[1] + 1; out->d_end = res[2] + 1;
-  }
+  SW_CUDA(h, cudaMemcpy(res, h->d_tb_result + 8, sizeof(res), cudaMemcpyDeviceToHost));
+  if (res[0] != se[0]) return fail(h, SW_E_CUDA, "traceback: box score differs from the full score");
+  out->q_begin = ib + res[3]; out->d_begin = jb + res[4];
+  out->q_end = ib + res[1] + 1; out->d_end = jb + res[2] + 1;
   out->n_ops = res[5];
   if (res[5] > ops_cap) return fail(h, SW_E_INVALID, "ops buffer too small (need " + std::to_string(res[5]) + ")");
   if (res[5] > 0) SW_CUDA(h, cudaMemcpy(ops, h->d_tb_ops, (size_t)res[5] * sizeof(uint32_t), cudaMemcpyDeviceToHost));
+  return SW_OK;
+}
+
+int sw_top_hits(sw_handle h, const int32_t* scores, int64_t n, int32_t k, int64_t* idx_out, int32_t* score_out) {
+  if (!h) return SW_E_INVALID;
+  if (k <= 0 || n <= 0) return SW_OK;
+  if (!scores || !idx_out || !score_out) return fail(h, SW_E_INVALID, "NULL buffer");
+  const int64_t kk = std::min<int64_t>(k, n);
+  const int ctas = topk_ctas(n);
+  auto al = [](size_t b) { return (b + 255) & ~(size_t)255; };
+  const size_t o_s = 0, o_hist = o_s + al((size_t)n * 4), o_cnt = o_hist + al(256 * 4),
+               o_tie = o_cnt + al(4), o_off = o_tie + al((size_t)ctas * 4), o_idx = o_off + al((size_t)ctas * 4),
+               o_sc = o_idx + al((size_t)kk * 8), total = o_sc + al((size_t)kk * 4);
+  int rc = grow(h, &h->d_tk, &h->tk_cap, total, "alloc top-hits scratch");
+  if (rc) return rc;
+  int32_t* d_s = reinterpret_cast<int32_t*>(h->d_tk + o_s);
+  uint32_t* d_hist = reinterpret_cast<uint32_t*>(h->d_tk + o_hist);
+  uint32_t* d_cnt = reinterpret_cast<uint32_t*>(h->d_tk + o_cnt);
+  uint32_t* d_tie = reinterpret_cast<uint32_t*>(h->d_tk + o_tie);
+  uint32_t* d_off = reinterpret_cast<uint32_t*>(h->d_tk + o_off);
+  int64_t* d_idx = reinterpret_cast<int64_t*>(h->d_tk + o_idx);
+  int32_t* d_sc = reinterpret_cast<int32_t*>(h->d_tk + o_sc);
+  SW_CUDA(h, cudaMemcpy(d_s, scores, (size_t)n * 4, cudaMemcpyHostToDevice));
+  // radix select: the k-th largest key, 8 bits per pass from the top
+  uint32_t prefix = 0, pmask = 0;
+  int64_t remaining = kk;   // how many keys equal to the prefix-so-far are still wanted
+  std::vector<uint32_t> hist(256);
+  const int hgrid = std::max(1, std::min(ctas, 4 * h->num_sms));
+  for (int shift = 24; shift >= 0; shift -= 8) {
+    SW_CUDA(h, cudaMemset(d_hist, 0, 256 * 4));
+    SW_CUDA(h, launch_tk_hist(d_s, n, shift, prefix, pmask, d_hist, hgrid, nullptr));
+    SW_CUDA(h, cudaMemcpy(hist.data(), d_hist, 256 * 4, cudaMemcpyDeviceToHost));
+    int64_t cum = 0;
+    int digit = 0;
+    for (int d = 255; d >= 0; --d) {
+      if (cum + hist[d] >= (uint64_t)remaining) { digit = d; break; }
+      cum += hist[d];
+    }
+    remaining -= cum;
+    prefix |= (uint32_t)digit << shift;
+    pmask |= 0xffu << shift;
+  }
+  const uint32_t thr = prefix;   // the k-th largest key; kk - remaining keys are above it
+  SW_CUDA(h, cudaMemset(d_cnt, 0, 4));
+  SW_CUDA(h, launch_tk_above(d_s, n, thr, d_idx, d_sc, d_cnt, d_tie, nullptr));
+  uint32_t above = 0;
+  SW_CUDA(h, cudaMemcpy(&above, d_cnt, 4, cudaMemcpyDeviceToHost));
+  if ((int64_t)above != kk - remaining) return fail(h, SW_E_CUDA, "top hits: selection count mismatch");
+  std::vector<uint32_t> ties((size_t)ctas), off((size_t)ctas);
+  SW_CUDA(h, cudaMemcpy(ties.data(), d_tie, (size_t)ctas * 4, cudaMemcpyDeviceToHost));
+  uint64_t acc = 0;
+  for (int b = 0; b < ctas; ++b) { off[(size_t)b] = (uint32_t)std::min<uint64_t>(acc, 0xffffffffu); acc += ties[(size_t)b]; }
+  SW_CUDA(h, cudaMemcpy(d_off, off.data(), (size_t)ctas * 4, cudaMemcpyHostToDevice));
+  SW_CUDA(h, launch_tk_ties(d_s, n, thr, d_off, (uint32_t)remaining, d_idx + above, d_sc + above, nullptr));
+  std::vector<int64_t> idx((size_t)kk);
+  std::vector<int32_t> sc((size_t)kk);
+  SW_CUDA(h, cudaMemcpy(idx.data(), d_idx, (size_t)kk * 8, cudaMemcpyDeviceToHost));
+  SW_CUDA(h, cudaMemcpy(sc.data(), d_sc, (size_t)kk * 4, cudaMemcpyDeviceToHost));
+  // the k selected hits, best first (score descending, index ascending)
+  std::vector<int64_t> ord((size_t)kk);
+  for (int64_t i = 0; i < kk; ++i) ord[(size_t)i] = i;
+  std::sort(ord.begin(), ord.end(), [&](int64_t a, int64_t b) {
+    return sc[(size_t)a] != sc[(size_t)b] ? sc[(size_t)a] > sc[(size_t)b] : idx[(size_t)a] < idx[(size_t)b];
+  });
+  for (int64_t i = 0; i < kk; ++i) { idx_out[i] = idx[(size_t)ord[(size_t)i]]; score_out[i] = sc[(size_t)ord[(size_t)i]]; }
   return SW_OK;
 }
 
@@ -1699,6 +1773,7 @@ void sw_destroy(sw_handle h) {
   for (auto& ss : h->stream_slot) ss.release();
   cudaFree(h->d_scores_tmp); cudaFree(h->d_batch_q);
   cudaFree(h->d_tb_dir); cudaFree(h->d_tb_scratch); cudaFree(h->d_tb_result); cudaFree(h->d_tb_ops);
+  cudaFree(h->d_tk);
   cudaFree(h->d_tb_query);
   if (h->fork) cudaEventDestroy(h->fork);
   if (h->gang_ev) cudaEventDestroy(h->gang_ev);

@@ -173,6 +173,19 @@ int scan_smem_bytes(int a_used, int cols_cta, int qcols);
 cudaError_t configure_scan_kernel(int smem_bytes, int ctas, int* max_clusters);
 cudaError_t launch_scan_pairs(const TParams& p, int items, int ctas, int smem_bytes, cudaStream_t st);
 
+// Top hits (sw_topk.cu): radix-select histogram passes, the keys above the threshold, the
+// threshold ties with the smallest indices (tie_off: exclusive prefix of the per-CTA tie counts).
+int topk_ctas(int64_t n);
+cudaError_t launch_tk_hist(const int32_t* s, int64_t n, int shift, uint32_t prefix, uint32_t pmask, uint32_t* hist,
+                           int grid, cudaStream_t st);
+cudaError_t launch_tk_above(const int32_t* s, int64_t n, uint32_t thr, int64_t* out_idx, int32_t* out_score,
+                            uint32_t* out_count, uint32_t* tie_count, cudaStream_t st);
+cudaError_t launch_tk_ties(const int32_t* s, int64_t n, uint32_t thr, const uint32_t* tie_off, uint32_t need,
+                           int64_t* out_idx, int32_t* out_score, cudaStream_t st);
+// Traceback, bounded memory: score + end cell (no directions), then the anchored reverse sweep
+// for the start cell; result[0..2] = score, end i, end j; [3..4] = start i, start j (-1: none).
+cudaError_t launch_tb_score_start(const uint8_t* q, int m, const uint16_t* dcols, int half, int n, const int8_t* W,
+                                  int A, int rho, int sigma, int* scratch, int* result, cudaStream_t st);
 // Traceback of one pair (sw_traceback.cu): dir = m*n bytes, scratch = 7*m ints, result = 6 ints.
 cudaError_t launch_traceback(const uint8_t* q, int m, const uint16_t* dcols, int half, int n, const int8_t* W, int A,
                              int rho, int sigma, uint8_t* dir, int* scratch, int* result, uint32_t* ops, int ops_cap,

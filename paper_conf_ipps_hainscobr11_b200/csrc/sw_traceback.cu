@@ -11,6 +11,16 @@
 // Ties prefer diagonal > E > F > 0 and extension > opening; the end cell is the maximum H,
 // first in (diagonal, row) order.
 // k_tb_walk: one thread follows the bytes back from the end cell and writes run-length ops.
+//
+// Bounded memory (round 2): the direction bytes are only written for the alignment's bounding
+// box.  (1) k_tb_fill without directions: the optimal score and its end cell (ie, je), O(m)
+// scratch.  (2) k_tb_start: Eq.(1) on the reversed prefixes q[ie..0] x d[je..0] ANCHORED at
+// (ie, je) (no 0 clamp, boundary -inf, the first cell a substitution): its value at (i, j) is the
+// best score of an alignment from (ie - i, je - j) to (ie, je) that starts with a substitution,
+// so a cell where it equals the optimum is the start (ib, jb) of an optimal local alignment (an
+// optimal one never starts or ends with a gap).  (3) k_tb_fill with directions on the box
+// q[ib..ie] x d[jb..je] only (its local optimum is the same score), and the walk.  Memory
+// (ie - ib + 1)(je - jb + 1) bytes instead of m n.
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -65,7 +75,7 @@ __global__ void __launch_bounds__(kTbThreads, 1)
       Hn[i] = h;
       En[i] = e;
       Fn[i] = f;
-      dir[(int64_t)i * n + j] = (uint8_t)(src | ((e_ext >= e_open) ? 4 : 0) | ((f_ext >= f_open) ? 8 : 0));
+      if (dir) dir[(int64_t)i * n + j] = (uint8_t)(src | ((e_ext >= e_open) ? 4 : 0) | ((f_ext >= f_open) ? 8 : 0));
       if (h > best || (h == best && (d < bd || (d == bd && i < bi)))) { best = h; bd = d; bi = i; }
     }
     __syncthreads();
@@ -88,6 +98,74 @@ __global__ void __launch_bounds__(kTbThreads, 1)
     result[0] = best;
     result[1] = best > 0 ? bi : -1;
     result[2] = best > 0 ? bd - bi : -1;
+  }
+}
+
+// (2) start cell: the anchored reverse sweep, anti-diagonals of the reversed prefixes; result
+// [3] = ib, [4] = jb of the first cell (diagonal, row order) whose value equals result[0]
+__global__ void __launch_bounds__(kTbThreads, 1)
+    k_tb_start(const uint8_t* __restrict__ q, const uint16_t* __restrict__ dcols, int half, const int8_t* __restrict__ W,
+               int A, int rho, int sigma, int* __restrict__ diag_scratch, int* __restrict__ result) {
+  const int best = result[0], ie = result[1], je = result[2];
+  if (best <= 0) {
+    if (threadIdx.x == 0) { result[3] = -1; result[4] = -1; }
+    return;
+  }
+  const int m = ie + 1, n = je + 1;   // reversed prefix: row i = q[ie - i], column j = d[je - j]
+  int* Hb[3] = {diag_scratch, diag_scratch + m, diag_scratch + 2 * m};
+  int* Eb[2] = {diag_scratch + 3 * m, diag_scratch + 4 * m};
+  int* Fb[2] = {diag_scratch + 5 * m, diag_scratch + 6 * m};
+  __shared__ int s_bd[kTbThreads / 32], s_bi[kTbThreads / 32];
+  __shared__ int s_found;
+  if (threadIdx.x == 0) s_found = 0;
+  __syncthreads();
+  int bd = 0x7fffffff, bi = 0x7fffffff;
+  const int shift = 8 * half;
+  for (int d = 0; d < m + n - 1; ++d) {
+    int* H2 = Hb[(d + 1) % 3];
+    int* H1 = Hb[(d + 2) % 3];
+    int* Hn = Hb[d % 3];
+    const int* E1 = Eb[(d + 1) & 1];
+    const int* F1 = Fb[(d + 1) & 1];
+    int* En = Eb[d & 1];
+    int* Fn = Fb[d & 1];
+    const int i0 = max(0, d - (n - 1)), i1 = min(m - 1, d);
+    for (int i = i0 + (int)threadIdx.x; i <= i1; i += blockDim.x) {
+      const int j = d - i;
+      // anchored boundary: H(-1, -1) = 0, every other H / E / F outside the prefix = -inf
+      const int hl = (j > 0) ? H1[i] : kNegInf;
+      const int el = (j > 0) ? E1[i] : kNegInf;
+      const int hu = (i > 0) ? H1[i - 1] : kNegInf;
+      const int fu = (i > 0) ? F1[i - 1] : kNegInf;
+      const int hd = (i > 0 && j > 0) ? H2[i - 1] : ((i == 0 && j == 0) ? 0 : kNegInf);
+      const int e = max(el - sigma, hl - rho);
+      const int f = max(fu - sigma, hu - rho);
+      const int a = (dcols[je - j] >> shift) & 0xff;
+      const int t = hd + (int)W[q[ie - i] * A + a];
+      const int h = max(max(t, e), max(f, kNegInf));
+      Hn[i] = h;
+      En[i] = max(e, kNegInf);
+      Fn[i] = max(f, kNegInf);
+      if (h == best && (d < bd || (d == bd && i < bi))) { bd = d; bi = i; }
+    }
+    __syncthreads();
+    // stop at the first diagonal that holds the start (all threads agree after the barrier)
+    if (bd != 0x7fffffff) s_found = 1;
+    __syncthreads();
+    if (s_found) break;
+  }
+  for (int o = 16; o >= 1; o >>= 1) {
+    const int od = __shfl_xor_sync(0xffffffffu, bd, o), oi = __shfl_xor_sync(0xffffffffu, bi, o);
+    if (od < bd || (od == bd && oi < bi)) { bd = od; bi = oi; }
+  }
+  const int w = threadIdx.x >> 5;
+  if ((threadIdx.x & 31) == 0) { s_bd[w] = bd; s_bi[w] = bi; }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (int k = 1; k < (int)(blockDim.x >> 5); ++k)
+      if (s_bd[k] < bd || (s_bd[k] == bd && s_bi[k] < bi)) { bd = s_bd[k]; bi = s_bi[k]; }
+    result[3] = ie - bi;          // ib
+    result[4] = je - (bd - bi);   // jb
   }
 }
 
@@ -144,6 +222,15 @@ __global__ void k_tb_walk(const uint8_t* __restrict__ dir, int m, int n, int* __
   result[3] = result[0] > 0 ? bi : -1;
   result[4] = result[0] > 0 ? bj : -1;
   result[5] = nops;
+}
+
+cudaError_t launch_tb_score_start(const uint8_t* q, int m, const uint16_t* dcols, int half, int n, const int8_t* W,
+                                  int A, int rho, int sigma, int* scratch, int* result, cudaStream_t st) {
+  k_tb_fill<<<1, kTbThreads, 0, st>>>(q, m, dcols, half, n, W, A, rho, sigma, nullptr, scratch, result);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  k_tb_start<<<1, kTbThreads, 0, st>>>(q, dcols, half, W, A, rho, sigma, scratch, result);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_traceback(const uint8_t* q, int m, const uint16_t* dcols, int half, int n, const int8_t* W, int A,

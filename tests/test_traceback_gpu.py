@@ -91,3 +91,53 @@ def test_align_errors():
         with pytest.raises(swp.SWError) as e:
             sw.align(5)
         assert e.value.status == swp.SW_E_INVALID
+
+
+def test_local_hit_in_long_sequence_bounded_box():
+    """A planted homologous window inside a 30,000-residue sequence: the bounded-memory traceback
+    (score + end cell, anchored reverse sweep for the start, directions for the bounding box only)
+    returns an optimal alignment inside the window's neighbourhood, rescored independently."""
+    rng = np.random.default_rng(21)
+    q = gen.make_query(300, seed=5)
+    d = rng.integers(0, 20, size=30000).astype(np.uint8)
+    win = q[40:260].copy()
+    mut = rng.random(win.size) < 0.25
+    win[mut] = rng.integers(0, 20, size=int(mut.sum()))
+    d[17000:17000 + win.size] = win
+    off = np.array([0, d.size], np.int64)
+    ref = oracle.scores(q, BLOSUM62, 10, 2, d, off)
+    with swp.SmithWaterman(q, BLOSUM62, 10, 2) as sw:
+        sw.load_db(d, off)
+        al = sw.align(0)
+    assert al["score"] == ref[0]
+    assert score_runs(q, d, BLOSUM62, 10, 2, al) == ref[0]
+    assert 16000 < al["d_begin"] < al["d_end"] < 18000
+
+
+def test_top_hits_match_numpy_order():
+    """sw_top_hits: the k largest scores (ties by the smaller index), best first, against a
+    numpy lexsort of the same array — real search output with many ties, negative and large
+    values, k beyond n."""
+    wl = gen.config("C1", n_override=20000)
+    q = wl.queries[0]
+    with swp.SmithWaterman(q, BLOSUM62, 10, 2) as sw:
+        sw.load_db(wl.db.residues, wl.db.offsets)
+        out = sw.search(3072)
+        cases = [out, np.array([5, -3, 7, 7, 2**31 - 1, -2**31, 0, 7], np.int32),
+                 np.random.default_rng(3).integers(-5, 5, size=100000).astype(np.int32)]
+        for arr in cases:
+            order = np.lexsort((np.arange(arr.size), -arr.astype(np.int64)))
+            for k in (1, 10, 1000, arr.size, arr.size + 5):
+                idx, val = sw.top_hits(arr, k)
+                kk = min(k, arr.size)
+                assert np.array_equal(idx, order[:kk]), (k, idx[:10], order[:10])
+                assert np.array_equal(val, arr[order[:kk]])
+        idx, val = sw.top_hits(out, 0)
+        assert idx.size == 0
+        # the top hits' alignments rescore to their search scores
+        idx, val = sw.top_hits(out, 5)
+        for i, v in zip(idx, val):
+            al = sw.align(int(i))
+            assert al["score"] == v
+            s, e = wl.db.offsets[i], wl.db.offsets[i + 1]
+            assert score_runs(q, wl.db.residues[s:e], BLOSUM62, 10, 2, al) == v
