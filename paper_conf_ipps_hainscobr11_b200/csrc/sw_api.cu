@@ -292,7 +292,6 @@ int make_plan(sw_handle h, int m, const Split& sp, Plan* pl, int force = -1,
   for (int i = 0; i < menu_size(); ++i) {
     const KernelConfig c = menu_entry(i);
     if (c.lane != 0 || (c.wide != 0) != h->wide) continue;
-    if (c.var != 0) continue;   // code variants: timed by the autotune beside their base entry
     ProfLayout lg, lt;
     int bytes = 0;
     main_layouts(c, m, A1, &lg, &lt, &bytes);
@@ -1239,23 +1238,6 @@ int autotune(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq,
       if (rc) return rc;
       if (getenv("SW_DEBUG_PLAN")) fprintf(stderr, "tune m=%d T=%d menu=%d %.3f ms\n", m, (int)Tk, c.second, ms);
       if (ms < best_ms) { best_ms = ms; best_i = c.second; }
-    }
-    // the winner's code variants (same configuration compiled differently, gen_menu.py)
-    if (best_i >= 0) {
-      const KernelConfig b = menu_entry(best_i);
-      for (int j = 0; j < menu_size(); ++j) {
-        const KernelConfig v = menu_entry(j);
-        if (j == best_i || v.var == 0 || v.lane != b.lane || v.G != b.G || v.Rs != b.Rs || v.Rl != b.Rl ||
-            v.threads != b.threads || v.wide != b.wide)
-          continue;
-        h->tune_force = j;
-        float ms = 0.f;
-        rc = time_search(k, Tk, &ms);
-        h->tune_force = -1;
-        if (rc) return rc;
-        if (getenv("SW_DEBUG_PLAN")) fprintf(stderr, "tune m=%d T=%d menu=%d (variant %d) %.3f ms\n", m, (int)Tk, j, v.var, ms);
-        if (ms < best_ms) { best_ms = ms; best_i = j; }
-      }
     }
     h->tuned[key] = best_i;
   }

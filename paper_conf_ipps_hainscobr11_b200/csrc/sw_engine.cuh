@@ -595,9 +595,7 @@ struct GsState {
 // MULTI = false: the query fits one strip (p.short_passes == 1), so there is no strip row
 // buffer: the first lane's top input is the constant boundary (H, F + rho) = (0, 0) and only
 // the residues go through the fetch ring (8 registers and 2 selects per step fewer).
-// V: code variant (same computation): 1 = the step's fetch issued after its rows, 2 = the
-// next step's shuffle ordered after H instead of F + rho
-template <class L, int R, bool MULTI, class CC, int V = 0>
+template <class L, int R, bool MULTI, class CC>
 __device__ __forceinline__ void group_stream(const SearchParams& p, const CC& c, const uint8_t* pbase,
                                              uint2* __restrict__ rb, volatile GsState* gs) {
   static_assert(R % 4 == 0 || R >= 12, "R < 12 must be a multiple of 4");
@@ -753,15 +751,13 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const CC& c,
       load_prof<R, CB, 32 * CB>(wlo, prow + off_lo);
       load_prof<R, CB, 32 * CB>(whi, prow + off_hi);
     }
-    if constexpr (V != 1) fetch(K);
+    fetch(K);
     uint32_t hup = x_hr, fs = x_f;
     cell_rows<L, R, CC::kWide>(e, t, wlo, whi, nrho, prho, nsig, hup, fs, best, dlt);
-    if constexpr (V == 1) fetch(K);
     y_hr = hup; y_f = fs; y_res = x_res;
     // keep the next step's residue shuffle (and so its profile loads) after this step's rows:
     // hoisting them would keep a second set of profile words live
-    if constexpr (V == 2) asm volatile("" : "+r"(y_res) : "r"(hup));
-    else asm volatile("" : "+r"(y_res) : "r"(fs));
+    asm volatile("" : "+r"(y_res) : "r"(fs));
     // unconditional for the storing lane: gap positions land in the slot's kGap leading
     // entries, stale positions past the segment beyond its columns; neither is ever read
     if (store_rb) rb[my_pos + K - kGap] = make_uint2(hup, fs);
@@ -812,7 +808,7 @@ __device__ __forceinline__ void group_stream(const SearchParams& p, const CC& c,
 // launcher compiles and picks 1 / 2 separately, so that each stream loop gets the kernel's
 // registers and instruction cache to itself (the two loops in one kernel shared one register
 // allocation: a change to one moved the other's timing by up to 2 %).
-template <class L, int G, int Rs, int Rl, int NT, bool WIDE = false, int GS = 0, int V = 0>
+template <class L, int G, int Rs, int Rl, int NT, bool WIDE = false, int GS = 0>
 __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
   constexpr int kWarps = NT / 32;
   extern __shared__ __align__(128) uint8_t smem[];
@@ -909,9 +905,9 @@ __global__ void __launch_bounds__(NT, 1) k_search(const SearchParams p) {
       __shared__ GsState sgs[kWarps];
       uint2* rbw = p.rb_group + (int64_t)(blockIdx.x * kWarps + warp) * p.rb_group_cols + 4;
       if constexpr (GS == 2) {
-        group_stream<L, Rs, true, ChainConstT<WIDE>, V>(p, c, smem + p.lg.off + lane * CBs, rbw, &sgs[warp]);
+        group_stream<L, Rs, true>(p, c, smem + p.lg.off + lane * CBs, rbw, &sgs[warp]);
       } else if constexpr (GS == 1) {
-        group_stream<L, Rs, false, ChainConstT<WIDE>, V>(p, c, smem + p.lg.off + lane * CBs, rbw, &sgs[warp]);
+        group_stream<L, Rs, false>(p, c, smem + p.lg.off + lane * CBs, rbw, &sgs[warp]);
       } else {
         if (p.short_passes > 1) group_stream<L, Rs, true>(p, c, smem + p.lg.off + lane * CBs, rbw, &sgs[warp]);
         else group_stream<L, Rs, false>(p, c, smem + p.lg.off + lane * CBs, rbw, &sgs[warp]);
@@ -1581,33 +1577,33 @@ cudaError_t configure_tmode(int smem_bytes, int* blocks_per_sm) {
 
 // G = 32 entries compile two kernels (GS = 1: single-strip group stream, GS = 2: multi-strip);
 // the 32-bit recompute (item_list) never reaches the group phase, so either serves it.
-template <class L, int G, int Rs, int Rl, int NT, bool WIDE, int V = 0>
+template <class L, int G, int Rs, int Rl, int NT, bool WIDE>
 cudaError_t launch_search_t(const SearchParams& p, int grid, int smem_bytes, cudaStream_t st) {
   if constexpr (G == 32) {
-    if (p.short_passes > 1) k_search<L, G, Rs, Rl, NT, WIDE, 2, V><<<grid, NT, smem_bytes, st>>>(p);
-    else k_search<L, G, Rs, Rl, NT, WIDE, 1, V><<<grid, NT, smem_bytes, st>>>(p);
+    if (p.short_passes > 1) k_search<L, G, Rs, Rl, NT, WIDE, 2><<<grid, NT, smem_bytes, st>>>(p);
+    else k_search<L, G, Rs, Rl, NT, WIDE, 1><<<grid, NT, smem_bytes, st>>>(p);
   } else {
     k_search<L, G, Rs, Rl, NT, WIDE><<<grid, NT, smem_bytes, st>>>(p);
   }
   return cudaGetLastError();
 }
 
-template <class L, int G, int Rs, int Rl, int NT, bool WIDE, int GS, int V = 0>
+template <class L, int G, int Rs, int Rl, int NT, bool WIDE, int GS>
 cudaError_t configure_one(int smem_bytes, int* blocks_per_sm) {
-  cudaError_t e = cudaFuncSetAttribute(k_search<L, G, Rs, Rl, NT, WIDE, GS, V>,
+  cudaError_t e = cudaFuncSetAttribute(k_search<L, G, Rs, Rl, NT, WIDE, GS>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search<L, G, Rs, Rl, NT, WIDE, GS, V>, NT,
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_search<L, G, Rs, Rl, NT, WIDE, GS>, NT,
                                                        smem_bytes);
 }
 
-template <class L, int G, int Rs, int Rl, int NT, bool WIDE, int V = 0>
+template <class L, int G, int Rs, int Rl, int NT, bool WIDE>
 cudaError_t configure_t(int smem_bytes, int* blocks_per_sm) {
   if constexpr (G == 32) {
     int b1 = 0, b2 = 0;
-    cudaError_t e = configure_one<L, G, Rs, Rl, NT, WIDE, 1, V>(smem_bytes, &b1);
+    cudaError_t e = configure_one<L, G, Rs, Rl, NT, WIDE, 1>(smem_bytes, &b1);
     if (e != cudaSuccess) return e;
-    e = configure_one<L, G, Rs, Rl, NT, WIDE, 2, V>(smem_bytes, &b2);
+    e = configure_one<L, G, Rs, Rl, NT, WIDE, 2>(smem_bytes, &b2);
     *blocks_per_sm = b1 < b2 ? b1 : b2;
     return e;
   } else {

@@ -90,8 +90,6 @@ struct KernelConfig {
   int Rl;
   int threads;   // CTA size (fewer threads for the register-heavy entries)
   int wide;      // 1: rho + max(w) > 127 variant (ChainConstT<true>, sw_engine.cuh)
-  int var;       // code variant of the group stream (0: base; sw_engine.cuh group_stream V): the
-                 // same computation compiled differently, timed by the autotune beside its base
 };
 
 // Launch one search; returns the CUDA error of the launch.
