@@ -153,6 +153,7 @@ struct sw_handle_s {
   // on each other, so two gang launches must never hold SMs at the same time; sw_engine.cuh
   // t_gang_item)
   cudaEvent_t gang_ev = nullptr;
+  cudaStream_t copy_st = nullptr;   // blocking API: per-query score copies as queries finish
   uint32_t gang_epoch = 0;        // tag epoch of the last gang launch (sw_engine.cuh run_pass GPU_FLAGS)
   // stats
   int64_t stat_long = 0, stat_short = 0, stat_launches = 0;
@@ -1352,7 +1353,8 @@ int sw_create(sw_handle* out, const uint8_t* query, int32_t query_len, const int
   if (cudaMalloc(&h->d_matrix, (size_t)alphabet_size * alphabet_size) != cudaSuccess ||
       cudaMemcpy(h->d_matrix, matrix, (size_t)alphabet_size * alphabet_size, cudaMemcpyHostToDevice) != cudaSuccess ||
       cudaEventCreateWithFlags(&h->fork, cudaEventDisableTiming) != cudaSuccess ||
-      cudaEventCreateWithFlags(&h->gang_ev, cudaEventDisableTiming) != cudaSuccess) {
+      cudaEventCreateWithFlags(&h->gang_ev, cudaEventDisableTiming) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&h->copy_st, cudaStreamNonBlocking) != cudaSuccess) {
     sw_destroy(h);
     return SW_E_CUDA;
   }
@@ -1580,8 +1582,31 @@ int sw_search_batch(sw_handle h, const uint8_t* queries, const int64_t* q_offset
   h->scores_tmp_cap = (int64_t)(cap / sizeof(int32_t));
   rc = sw_search_batch_async(h, queries, q_offsets, num_queries, h->d_scores_tmp, length_threshold, nullptr);
   if (rc) return rc;
-  if (need > 0)
+  // each query's scores are final at its ev[2] (after its 32-bit recompute): copy them as the
+  // queries finish, on a stream of their own, so the copies overlap the queries still running
+  // (the caller's stream waits for every query; a copy there would wait for the last one)
+  const int64_t ns = h->db->n_seqs;
+  if (need > 0 && (int)h->ev.size() >= kEvPerQuery * num_queries) {
+    std::vector<char> copied((size_t)num_queries, 0);
+    for (int left = num_queries; left > 0;) {
+      int progressed = 0;
+      for (int k = 0; k < num_queries; ++k) {
+        if (copied[(size_t)k]) continue;
+        const cudaError_t q = cudaEventQuery(h->ev[(size_t)kEvPerQuery * k + 2]);
+        if (q == cudaErrorNotReady) continue;
+        if (q != cudaSuccess) return cuda_fail(h, q, "query completion");
+        SW_CUDA(h, cudaMemcpyAsync(scores_out + (int64_t)k * ns, h->d_scores_tmp + (int64_t)k * ns,
+                                   (size_t)ns * sizeof(int32_t), cudaMemcpyDeviceToHost, h->copy_st));
+        copied[(size_t)k] = 1;
+        --left;
+        ++progressed;
+      }
+      if (!progressed) std::this_thread::yield();
+    }
+    SW_CUDA(h, cudaStreamSynchronize(h->copy_st));
+  } else if (need > 0) {
     SW_CUDA(h, cudaMemcpy(scores_out, h->d_scores_tmp, (size_t)need * sizeof(int32_t), cudaMemcpyDeviceToHost));
+  }
   SW_CUDA(h, cudaDeviceSynchronize());
   return SW_OK;
 }
@@ -1777,6 +1802,7 @@ void sw_destroy(sw_handle h) {
   cudaFree(h->d_tb_query);
   if (h->fork) cudaEventDestroy(h->fork);
   if (h->gang_ev) cudaEventDestroy(h->gang_ev);
+  if (h->copy_st) cudaStreamDestroy(h->copy_st);
   if (h->h_ovf) cudaFreeHost(h->h_ovf);
   delete h;
 }

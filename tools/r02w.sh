@@ -1,5 +1,4 @@
-for lib in build/old/libsw_b200.so ""; do
-  for m in 144 567; do SW_LIB=$lib timeout 60 python tools/profile_long.py $m 3073 3 C3 | tail -1 | sed "s|^|[lib=$lib] |"; done
-  for T in 3072 1172 512; do SW_LIB=$lib timeout 90 python tools/profile_long.py 567 $T 3 C2 | tail -1 | sed "s|^|[lib=$lib] |"; done
-  SW_LIB=$lib SW_T_PACKED=0 timeout 60 python tools/profile_long.py 567 3072 3 C2 | tail -1 | sed "s|^|[lib=$lib packed0] |"
-done > gpurun_out/r02w.txt 2>&1
+mkdir -p gpurun_out/w1
+timeout 900 python -m pytest tests/test_abi_gpu.py tests/test_parity_full_gpu.py tests/test_traceback_gpu.py -q -p no:cacheprovider -x 2>&1 | tail -2
+for i in 1 2; do timeout 900 python bench.py --no-cpu-baseline --no-stream > gpurun_out/w1/bench$i.jsonl 2> gpurun_out/w1/bench$i.err; python -c "
+import json; d=json.loads(open('gpurun_out/w1/bench$i.jsonl').read().strip().splitlines()[-1]); print(d['value'], d['e2e']['value'], d['roofline']['frac'], d['parity']['mismatches'], d['auto_threshold']['value'])"; done
