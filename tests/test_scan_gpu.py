@@ -114,3 +114,18 @@ def test_scan_repeated_and_batched():
     finally:
         os.environ.pop("SW_LONG_MODE", None)
         os.environ.pop("SW_SCAN", None)
+
+
+def test_scan_chosen_automatically_for_an_outlier_pair():
+    """No SW_SCAN: the planner scans pair 0 on its own when it is an outlier (its time alone
+    bounds the launch and it has >= 1.5x the next pair's columns) — a 64,000 / 60,000-residue
+    pair beside 3-8k sequences — with gangs / teams for the rest, the T-mode kernel as a
+    programmatic dependent launch behind the scan."""
+    rng = np.random.default_rng(99)
+    lens = np.concatenate([[64000, 60000], rng.integers(3073, 8000, size=60), rng.integers(0, 300, size=30)])
+    db = gen.build_database(lens.astype(np.int64), 123, None)
+    for m in (300, 567):
+        q = gen.make_query(m, seed=m + 7)
+        ref = oracle.scores(q, BLOSUM62, 10, 2, db.residues, db.offsets)
+        out, _ = _search(q, BLOSUM62, 10, 2, db, 3072, {"SW_LONG_MODE": "t"})
+        _check(out, ref, db, f"auto scan m={m}")
