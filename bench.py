@@ -507,7 +507,7 @@ def bench_ours(args, rank, world, local_rank):
                    **({"c5_shards": max(world, int(os.environ.get("C5_SHARDS", "64")))} if args.config == "C5" else {})},
         "clocks": clk,
         "e2e": {"value": round(e2e_gcups, 2), "unit": "GCUPS", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-                "api": "sw_search_batch (blocking, host buffers; DB resident as in PAPER.md L32)"},
+                "api": "sw_search_batch (blocking; queries from host memory, scores copied per query as it finishes into a pinned host buffer reused across steps; DB resident as in PAPER.md L32)"},
         "gpu_launches": int(st["launches"]) * args.steps,
         "roofline": roof,
         "parity": parity,
