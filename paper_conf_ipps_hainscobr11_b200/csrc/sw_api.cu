@@ -48,6 +48,7 @@ struct QuerySlot {
   cudaStream_t scan = nullptr;     // row-scan cluster launches (sw_scan.cu), beside the T-mode launch
   cudaEvent_t scan_fork = nullptr, scan_done = nullptr;
   int scan_smem = -1;              // the row-scan kernel's configured dynamic shared memory
+  uint32_t scan_ctas_ok = 0;       // cluster sizes checked for that configuration (bit K)
   cudaEvent_t done = nullptr;
   cudaEvent_t fork = nullptr, join = nullptr;
 };
@@ -689,7 +690,7 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
     }
     TParams t{};
     std::vector<int32_t> h_gang_base;   // per-gang CTA slot offsets (uploaded with the gang scratch)
-    std::vector<int> scan_cols;         // row-scan items [0, size): columns per CTA
+    std::vector<int> scan_ctas, scan_cols;   // row-scan items [0, size): cluster size, columns per CTA
     t.matrix = h->d_matrix;
     t.A = h->A;
     t.rho = h->rho16;
@@ -778,35 +779,54 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
         t_thr /= nw;
         const bool hidden = (double)sp.short_cols > 0.5 * (double)sp.long_cols;
         int K = 0, items = 0;
-        // Row scan (sw_scan.cu): the longest pairs of a launch
-        // that is not hidden run one query row per cluster time step instead of strip pipelines
-        // (their wavefront bound): a prefix of the long pairs (longest first) with at least
-        // kScanMinCols columns and at most kScanCtas x kScanCols, each on a cluster of kScanCtas
-        // CTAs, all in one launch.  SW_SCAN=0 disables it, SW_SCAN=N forces it for every
-        // long pair of >= N columns (tests, probes).
+        // Row scan (sw_scan.cu): in a launch that is not
+        // hidden, a prefix of the longest pairs runs one query row per step on clusters of
+        // K = ceil(ncols / kScanCols) CTAs.  The prefix length j minimises the launch estimate
+        //   max(the scans: (qcols + K) x kScanRowSteps steps, all concurrent,
+        //       the longest remaining wavefront (S - 1) lag + qsteps,
+        //       the remaining pairs' throughput time on the SMs the clusters leave),
+        // j = 0 being today's plan; at most 3/4 of the SMs in clusters.  SW_SCAN=0 disables it,
+        // SW_SCAN=N forces it for the (up to 4) longest pairs of >= N columns.
         {
           int scan_min = kScanMinCols;
           bool forced = false;
           if (const char* f = getenv("SW_SCAN"); f && *f) { scan_min = atoi(f); forced = scan_min > 0; }
+          double row_steps = kScanRowSteps;
+          if (const char* f = getenv("SW_SCAN_ROW_STEPS")) row_steps = atof(f);   // probes
+          int sms = 0;
           if (scan_min > 0 && (forced || !hidden) && !h->wide && a_used + 1 <= kScanMaxLetters) {
+            std::vector<double> thr_tail(n_long + 1, 0.0);   // throughput steps of pairs [pp, n_long)
+            for (int pp = n_long - 1; pp >= 0; --pp) {
+              const double S = std::ceil((double)h->db->h_pair_ncols[pp] / spos);
+              thr_tail[pp] = thr_tail[pp + 1] + S * qsteps / util(W, S, false) / nw;
+            }
+            auto wavefront = [&](int pp) {
+              return pp < n_long ? (std::ceil((double)h->db->h_pair_ncols[pp] / spos) - 1.0) * lag + qsteps : 0.0;
+            };
+            double best = std::max(wavefront(0), thr_tail[0]), scan_t = 0.0;
+            int best_j = 0;
+            std::vector<int> ks, cs;
             for (int pp = 0; pp < n_long && pp < (forced ? 4 : kMaxScanItems); ++pp) {
               const int nc = h->db->h_pair_ncols[pp];
-              if (nc < scan_min || nc > kScanCtas * kScanCols) break;
-              if (!forced) {
-                // only an outlier: a pair whose time alone bounds the launch (a gang candidate)
-                // AND is >= 1.5x the next pair's columns.  The scan computes ~2.7x fewer cells
-                // per SM than the team stream (C2 top pair, query 567: 0.418 ms on 16 SMs vs
-                // 0.693 ms as a gang), so for a tail of similar pairs (C2 at T = 3072: 22 pairs
-                // of 16-35k columns) it only takes SMs from the others: 0.98 vs 0.92 ms
-                const double S = std::ceil((double)nc / spos);
-                if (item_time(S >= t.big_strips ? t_warps : W, S) <= 1.15 * t_thr) break;
-                if (pp + 1 < n_long && nc < 1.5 * h->db->h_pair_ncols[pp + 1]) break;
-              }
-              scan_cols.push_back(scan_cols_cta(nc, kScanCtas));
+              if (nc < scan_min || nc > kScanMaxCtas * kScanCols) break;
+              const int Kc = (nc + kScanCols - 1) / kScanCols;
+              if (!forced && sms + Kc > 3 * h->num_sms / 4) break;
+              sms += Kc;
+              ks.push_back(Kc);
+              cs.push_back(scan_cols_cta(nc, Kc));
+              scan_t = std::max(scan_t, (qcols + Kc) * row_steps);
+              const double left = 1.0 - (double)sms / h->num_sms;
+              const double est = std::max({scan_t, wavefront(pp + 1), thr_tail[pp + 1] / left});
+              if (forced || est < 0.97 * best) { best = std::min(best, est); best_j = pp + 1; }
             }
+            scan_ctas.assign(ks.begin(), ks.begin() + best_j);
+            scan_cols.assign(cs.begin(), cs.begin() + best_j);
+            sms = 0;
+            for (int k2 : scan_ctas) sms += k2;
           }
           if (getenv("SW_DEBUG_PLAN") && !scan_cols.empty())
-            fprintf(stderr, "tmode scan items=%zu (first %d columns per CTA)\n", scan_cols.size(), scan_cols[0]);
+            fprintf(stderr, "tmode scan items=%zu (%d SMs; first %d CTAs x %d columns)\n", scan_cols.size(), sms,
+                    scan_ctas[0], scan_cols[0]);
         }
         // gangs for the long pairs after the scanned ones (gang gi = pair scan items + gi)
         const int s0 = (int)scan_cols.size();
@@ -914,15 +934,28 @@ int enqueue_query(sw_handle h, QuerySlot& s, const uint8_t* d_q, int m, uint32_t
       // launched on another stream, the T-mode kernel's persistent CTAs could take every SM
       // first and leave no GPC free for a 16-CTA cluster until they finish (measured: the two
       // kernels serialised).  The T-mode queue starts after the scanned pairs (t.q0).
-      const int ssmem = scan_smem_bytes(a_used, scan_cols[0], qcols);
-      if (s.scan_smem != ssmem) {
-        int maxc = 0;
-        cudaError_t e = configure_scan_kernel(ssmem, kScanCtas, &maxc);
-        if (e != cudaSuccess) return cuda_fail(h, e, "configure row-scan kernel");
-        if (maxc < 1) return fail(h, SW_E_UNSUPPORTED, "row-scan cluster cannot be placed");
-        s.scan_smem = ssmem;
+      // one launch per cluster size (sizes are non-increasing along the longest-first items),
+      // each behind the previous one as a programmatic dependent launch
+      int smax = 0;
+      for (size_t i = 0; i < scan_cols.size(); ++i) smax = std::max(smax, scan_smem_bytes(a_used, scan_cols[i], qcols));
+      bool pdl = false;
+      for (size_t i0 = 0; i0 < scan_cols.size();) {
+        size_t i1 = i0;
+        while (i1 < scan_cols.size() && scan_ctas[i1] == scan_ctas[i0]) ++i1;
+        const int K = scan_ctas[i0];
+        if (s.scan_smem != smax || (s.scan_ctas_ok & (1u << K)) == 0) {
+          int maxc = 0;
+          cudaError_t e = configure_scan_kernel(smax, K, &maxc);
+          if (e != cudaSuccess) return cuda_fail(h, e, "configure row-scan kernel");
+          if (maxc < 1) return fail(h, SW_E_UNSUPPORTED, "row-scan cluster cannot be placed");
+          if (s.scan_smem != smax) s.scan_ctas_ok = 0;
+          s.scan_smem = smax;
+          s.scan_ctas_ok |= 1u << K;
+        }
+        SW_CUDA(h, launch_scan_pairs(t, (int)i0, (int)(i1 - i0), K, smax, tst, pdl));
+        pdl = true;
+        i0 = i1;
       }
-      SW_CUDA(h, launch_scan_pairs(t, (int)scan_cols.size(), kScanCtas, ssmem, tst));
     }
     SW_CUDA(h, launch_tmode(t, t_grid, t_smem, tst, false, !scan_cols.empty()));
     SW_CUDA(h, cudaEventRecord(ev[4], tst));

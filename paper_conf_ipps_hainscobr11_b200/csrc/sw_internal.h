@@ -158,20 +158,22 @@ cudaError_t configure_tmode_kernel(int smem_bytes, int* blocks_per_sm, bool wide
                                    bool packed = false);
 cudaError_t launch_qpair(uint16_t* out, const uint8_t* q, int m, int n, uint32_t qmask, cudaStream_t st);
 
-// Row scan (sw_scan.cu): long pairs [0, items) on one cluster of `ctas` CTAs each (one launch),
-// ceil(ncols / ctas) columns per CTA rounded up to 128 (<= kScanCols); the scores are emitted
-// like k_search_t's (emit_t).
+// Row scan (sw_scan.cu): long pairs on clusters of ceil(ncols / kScanCols) CTAs (<= 16), the
+// pairs of one cluster size in one launch; ceil(ncols / K) columns per CTA rounded up to 128
+// (<= kScanCols); the scores are emitted like k_search_t's (emit_t).
 constexpr int kScanThreads = 1024;
 constexpr int kScanC = 4;
 constexpr int kScanCols = kScanThreads * kScanC;
-constexpr int kScanCtas = 16;            // cluster size (non-portable, <= 16)
+constexpr int kScanMaxCtas = 16;         // cluster size limit (non-portable above 8)
 constexpr int kScanMaxLetters = 26;      // (A_used + 1) x 2 x cols_cta bytes of tables + the query
-constexpr int kScanMinCols = 16384;      // pairs from 1024 columns per CTA up
-constexpr int kMaxScanItems = 1;      // each takes 16 SMs from the team stream (C2 query 567, T = 3072: 4 items 1.32 ms, 1 item see DESIGN)
+constexpr int kScanMinCols = 16384;
+constexpr int kMaxScanItems = 32;
+constexpr double kScanRowSteps = 10.0;   // a scan row's time in strip steps, calibrated on C2 long sets (queries 144-729, r02_row_scan.txt)
 int scan_cols_cta(int ncols, int ctas);
 int scan_smem_bytes(int a_used, int cols_cta, int qcols);
 cudaError_t configure_scan_kernel(int smem_bytes, int ctas, int* max_clusters);
-cudaError_t launch_scan_pairs(const TParams& p, int items, int ctas, int smem_bytes, cudaStream_t st);
+cudaError_t launch_scan_pairs(const TParams& p, int item0, int items, int ctas, int smem_bytes, cudaStream_t st,
+                              bool pdl);
 
 // Top hits (sw_topk.cu): radix-select histogram passes, the keys above the threshold, the
 // threshold ties with the smallest indices (tie_off: exclusive prefix of the per-CTA tie counts).

@@ -72,18 +72,18 @@ __device__ __forceinline__ uint32_t ld_cl32(uint32_t a) {   // (the right CTA's 
 // One launch runs all row-scan items: cluster c (CTAs [c K, c K + K)) takes long pair c, with
 // cols_cta = ceil(ncols / K) rounded up to 128 columns (the dynamic shared memory is sized for
 // pair 0, the longest).
-__global__ void __launch_bounds__(kScanThreads, 1) k_scan_pair(const TParams p) {
+__global__ void __launch_bounds__(kScanThreads, 1) k_scan_pair(const TParams p, int item0) {
   using L = LaneS16x2;
   extern __shared__ __align__(16) uint8_t tab[];   // [(a * 2 + s) * cols_cta + j]: w, int8; then the query
   __shared__ unsigned long long s_eo[32][kRing];   // (row + 1) << 32 | E + rho entering warp w's first column
   __shared__ unsigned long long s_hl[32][kRing];   // (row + 1) << 32 | H of the left neighbour's last column
   __shared__ uint32_t s_cons[32];                  // rows consumed, per receiver
-  __shared__ uint32_t s_best[kScanCtas];
+  __shared__ uint32_t s_best[kScanMaxCtas];
   __shared__ uint32_t s_red[32];
   __shared__ uint8_t s_real[33];
   cg::cluster_group cl = cg::this_cluster();
   const int k = (int)cl.block_rank(), K = (int)cl.num_blocks();
-  const int item = (int)blockIdx.x / K;
+  const int item = item0 + (int)blockIdx.x / K;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int ncols = p.pair_ncols[item];
   const int cols_cta = ((ncols + K - 1) / K + 32 * kScanC - 1) / (32 * kScanC) * (32 * kScanC);
@@ -254,7 +254,10 @@ cudaError_t configure_scan_kernel(int smem_bytes, int ctas, int* max_clusters) {
   return cudaOccupancyMaxActiveClusters(max_clusters, k_scan_pair, &cfg);
 }
 
-cudaError_t launch_scan_pairs(const TParams& p, int items, int ctas, int smem_bytes, cudaStream_t st) {
+// items [item0, item0 + items) on clusters of `ctas` CTAs; pdl: programmatic dependent launch
+// behind the previous scan launch on the stream (its clusters trigger once resident)
+cudaError_t launch_scan_pairs(const TParams& p, int item0, int items, int ctas, int smem_bytes, cudaStream_t st,
+                              bool pdl) {
   cudaLaunchConfig_t cfg = {};
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeClusterDimension;
@@ -267,7 +270,14 @@ cudaError_t launch_scan_pairs(const TParams& p, int items, int ctas, int smem_by
   cfg.stream = st;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, k_scan_pair, p);
+  cudaLaunchAttribute attr2[2] = {attr[0], {}};
+  if (pdl) {
+    attr2[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr2[1].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr2;
+    cfg.numAttrs = 2;
+  }
+  return cudaLaunchKernelEx(&cfg, k_scan_pair, p, item0);
 }
 
 }  // namespace swb
