@@ -1262,8 +1262,9 @@ int autotune(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq,
     if (ranked.size() > (size_t)kTuneTop) ranked.resize(kTuneTop);
     rc = fork();
     if (rc) return rc;
-    float best_ms = 1e30f;
-    int best_i = -1;
+    // one timed search per candidate, then the two fastest again (min of two): a single
+    // disturbed timing once kept a 4 % slower entry for a whole session (query 2504 on C2)
+    std::vector<std::pair<float, int>> timed;
     for (const auto& c : ranked) {
       h->tune_force = c.second;
       float ms = 0.f;
@@ -1271,9 +1272,20 @@ int autotune(sw_handle h, const uint8_t* d_queries, const int64_t* qoff, int nq,
       h->tune_force = -1;
       if (rc) return rc;
       if (getenv("SW_DEBUG_PLAN")) fprintf(stderr, "tune m=%d T=%d menu=%d %.3f ms\n", m, (int)Tk, c.second, ms);
-      if (ms < best_ms) { best_ms = ms; best_i = c.second; }
+      timed.push_back({ms, c.second});
     }
-    h->tuned[key] = best_i;
+    std::sort(timed.begin(), timed.end());
+    for (size_t j = 0; j < std::min<size_t>(2, timed.size()); ++j) {
+      h->tune_force = timed[j].second;
+      float ms = 0.f;
+      rc = time_search(k, Tk, &ms);
+      h->tune_force = -1;
+      if (rc) return rc;
+      if (getenv("SW_DEBUG_PLAN")) fprintf(stderr, "tune m=%d T=%d menu=%d %.3f ms (again)\n", m, (int)Tk, timed[j].second, ms);
+      timed[j].first = std::min(timed[j].first, ms);
+    }
+    std::sort(timed.begin(), timed.end());
+    h->tuned[key] = timed.empty() ? -1 : timed[0].second;
   }
   if (forked) SW_CUDA(h, cudaStreamSynchronize(h->slots[0].stream));
   h->stat_long = h->stat_short = h->stat_launches = 0;
