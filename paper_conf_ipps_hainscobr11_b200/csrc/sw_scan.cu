@@ -11,14 +11,15 @@
 //   E[j+1] = max(E[j] - sigma, H[j] - rho) = max(E[j] - sigma', Ht[j] - rho),  sigma' = min(sigma, rho)
 // (H[j] = max(Ht[j], E[j]) and E[j] - rho <= E[j] - sigma' — exact, also for sigma > rho), so
 // a run of c columns maps its entering E to max(E - c sigma', b) and these maps compose:
-// (a1, b1) then (a2, b2) = (a1 + a2, max(b1 - a2, b2)).  A thread owns kScanC = 4 columns, a
-// warp and then the CTA scan the maps (shuffles, one barrier), and the row's entering E of a
-// CTA comes from the CTA on its left: CTA k of the cluster processes row t - k at time step t
-// (a wavefront over the cluster), so that value — and the left column's H for the next row's
-// diagonal — was produced one time step earlier and is handed over through distributed shared
-// memory, with one cluster barrier per time step.  Values are s16x2 (the pair's two sequences)
-// with the overflow flag of the other kernels; E + rho >= 0 always (E >= H - rho >= -rho), so
-// the scan runs on E + rho with the offsets clamped to 32767 and never wraps.
+// (a1, b1) then (a2, b2) = (a1 + a2, max(b1 - a2, b2)).  A lane owns kScanC = 4 columns and a
+// warp scans its 32 lanes' maps with shuffles; the warps of the whole cluster then form one
+// pipeline along the row (below): a warp needs only the E entering its first column from its
+// left neighbour, and rows i, i+1, ... are in flight along the pipeline at once.  Values are
+// s16x2 (the pair's two sequences) with the overflow flag of the other kernels; E + rho >= 0
+// always (E >= H - rho >= -rho), so the scan runs on E + rho with the offsets clamped to 32767
+// and never wraps.  (Measured and replaced: a CTA-wide scan per row with one cluster barrier
+// per time step, 2.5-3x slower; release / acquire hand-off flags, which compile to
+// MEMBAR.ALL.GPU per row here, 3.5x slower — profiles/r02_row_scan.txt.)
 #include <cooperative_groups.h>
 
 #include "sw_engine.cuh"
